@@ -1,0 +1,179 @@
+/* sfs.h — C ABI of libsfs: B200-native featurisation, format conversion, per-format SpMV and
+ * format-race labelling of sparse matrices.
+ *
+ * Paper: Dhandhania, Deodhar, Pogorelov, Biswas, Langguth, "Explaining the Performance of Supervised
+ * and Semi-Supervised Methods for Automated Sparse Matrix Format Selection", ICPP Workshops '21
+ * (/root/reference/PAPER.md; "P:L<n>" = its line n).  The library implements the benchmarking /
+ * labelling pass the paper identifies as the cost of supervised training (§1, §5.1,
+ * P:L331–333 §5.4): for each matrix, the Table-1 features, conversion of the CSR input
+ * into every candidate format (§2.1, P:L331 step ii), timed SpMV y = A·x in each format
+ * ("average over 100 trials" P:L217, step iii of P:L331) and the fastest format as label
+ * (§1).  Readings where the paper is silent are DESIGN.md §"Readings" (Q1–Q18).
+ *
+ * Conventions (every function):
+ *  - All array pointers are DEVICE pointers unless a field says otherwise (sfs_csr.mem).
+ *  - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  All work is
+ *    stream-ordered on it.  Only functions that return host results synchronize it (marked
+ *    "syncs").  sfs_spmv never synchronizes.
+ *  - No C++ exception crosses the ABI.  Every call returns an sfs_status; CUDA errors map to
+ *    SFS_ERR_CUDA with the detail in sfs_last_error() (thread-local string).
+ *  - Indices are int32: nnz >= 2^31 or nrows/ncols >= 2^31 gives SFS_ERR_UNSUPPORTED.  Size
+ *    features are int64 (an inadmissible ELL can have > 2^31 slots).
+ *  - x, y and the matrix values share one dtype (fp32 or fp64).
+ *  - Input CSR must be canonical (Q16): row_ptr[0] = 0, row_ptr non-decreasing,
+ *    row_ptr[nrows] = nnz, 0 <= col < ncols, columns strictly increasing within a row.  Empty
+ *    rows and explicit zeros are allowed.  Checked on the device; violation -> SFS_ERR_INVALID_CSR.
+ *  - Library-owned buffers (sfs_matrix) come from the allocator hook (default: a CUDA
+ *    stream-ordered memory pool) and live until sfs_matrix_free.
+ *  - GPU only: without a CUDA device every compute call returns SFS_ERR_CUDA.  There is no CPU
+ *    fallback.
+ */
+#ifndef SFS_H
+#define SFS_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  SFS_OK = 0,
+  SFS_ERR_INVALID_ARG = -1,
+  SFS_ERR_INVALID_CSR = -2,
+  SFS_ERR_INADMISSIBLE = -3, /* ELL / DIA past the fill guard (Q11; cf. CUSP size failures P:L194) */
+  SFS_ERR_OOM = -4,
+  SFS_ERR_CUDA = -5,
+  SFS_ERR_UNSUPPORTED = -6,
+  SFS_ERR_NOT_RUN = -7       /* format excluded by formats_mask */
+} sfs_status;
+
+/* Formats of P:L73 (§2.1) raced by the paper plus DIA.  The enum order is the
+   tie-break order of the label rule (Q14). */
+typedef enum { SFS_CSR = 0, SFS_COO = 1, SFS_ELL = 2, SFS_HYB = 3, SFS_DIA = 4, SFS_NFMT = 5 } sfs_format;
+typedef enum { SFS_F32 = 0, SFS_F64 = 1 } sfs_dtype;
+typedef enum { SFS_MEM_DEVICE = 0, SFS_MEM_HOST = 1 } sfs_memspace;
+
+/* A borrowed CSR matrix (caller-owned; never freed or written by the library).
+   mem = SFS_MEM_HOST: row_ptr/col_idx/values (and x) are host pointers (pinned for speed); the
+   library copies them to the device inside the call (this is the end-to-end path). */
+typedef struct {
+  int64_t nrows, ncols, nnz;
+  const int32_t *row_ptr; /* nrows+1 */
+  const int32_t *col_idx; /* nnz */
+  const void *values;     /* nnz of float (SFS_F32) or double (SFS_F64) */
+  int32_t dtype;          /* sfs_dtype */
+  int32_t mem;            /* sfs_memspace of the four pointers */
+  const void *x;          /* sfs_label_corpus only: race input vector (ncols); NULL = all ones */
+} sfs_csr;
+
+/* Table-1 features, host struct.  Integer features are exact; each double is one
+   fixed fp64 expression of exact integer aggregates (DESIGN.md §"Readings" Q1–Q9). */
+typedef struct {
+  int64_t nrows, ncols, nnz, nnz_min, nnz_max, csr_max, ell_size, hyb_k, hyb_ell_size, hyb_coo,
+      hyb_ell_nnz, diagonals, dia_size;
+  double nnz_frac, nnz_mu, nnz_sig, max_mu, mu_min, sig_lower, sig_higher, hyb_ell_frac, dia_frac,
+      ell_frac;
+  uint32_t admissible_mask; /* bit f set iff format f is admissible (Q11) */
+  int32_t csr_variant;      /* CSR kernel the library picks for this matrix (Q17): 0 vector, 1 merge */
+} sfs_features_t;
+
+typedef struct sfs_matrix_ *sfs_matrix; /* opaque, library-owned */
+
+/* Physical layout of a converted matrix (read-only device pointers, for tests / inspection).
+   pitch P = ceil(nrows/32)*32.  ptr[] by format:
+     CSR: 0 row_ptr, 1 col, 2 val                       (borrowed from the caller for device input)
+     COO: 0 row, 1 col, 2 val                           (nnz each, CSR order)
+     ELL: 0 col[width*P], 1 val[width*P]                column-major slab: entry (r, j) at j*P + r;
+                                                        padding col = -1, val = +0 (Q10)
+     HYB: 0 ell col, 1 ell val (width = hyb_k, as ELL), 2 coo row, 3 coo col, 4 coo val (coo_nnz)
+     DIA: 0 offsets[ndiag] (ascending), 1 val[ndiag*P]  entry (d, r) at d*P + r, +0 where absent */
+typedef struct {
+  int32_t fmt, dtype;
+  int64_t nrows, ncols, nnz, pitch, width, ndiag, coo_nnz;
+  const void *ptr[6];
+  int64_t bytes;     /* device bytes owned by the handle */
+  int32_t variant;   /* CSR kernel variant (Q17) */
+} sfs_layout_t;
+
+/* Race options (mean of 100 trials).  sfs_default_opts fills the DESIGN.md defaults. */
+typedef struct {
+  int32_t reps;          /* timed SpMVs per format (100) */
+  int32_t warmup;        /* untimed SpMVs before timing (5) (Q13) */
+  uint32_t formats_mask; /* formats to race (0x1F = all five; 0x0F = the paper's four) */
+  int32_t cold;          /* 0 = back-to-back reps (labels); 1 = flush L2 before every rep */
+  double max_fill;       /* Q11 ELL/DIA guard: slots <= max(trunc(max_fill*nnz), fill_slack) (3.0) */
+  int64_t fill_slack;    /* (1<<20) */
+  double hyb_rel_speed;  /* Q6 HYB width rule (3.0) */
+  int64_t hyb_breakeven; /* (4096) */
+  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge */
+  int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (1) */
+} sfs_race_opts;
+
+/* Result of racing one matrix. */
+typedef struct {
+  int32_t label;            /* argmin t_spmv over run formats, ties to the lowest id (Q14); -1 if none */
+  uint32_t admissible_mask; /* Q11 */
+  int32_t matrix_status;    /* SFS_OK or the error that stopped this matrix (e.g. INVALID_CSR) */
+  int32_t csr_variant;
+  float t_spmv_us[SFS_NFMT];    /* mean device time of one SpMV (CUDA events around `reps`) */
+  float t_convert_us[SFS_NFMT]; /* device time of CSR -> f (0 for CSR) */
+  int32_t status[SFS_NFMT];     /* SFS_OK, SFS_ERR_INADMISSIBLE, SFS_ERR_NOT_RUN, SFS_ERR_OOM, ... */
+  int64_t bytes[SFS_NFMT];      /* algorithmic bytes of one SpMV in format f */
+  float t_features_us;          /* device time of the feature pass (batched: 0 if not measured) */
+} sfs_label_t;
+
+void sfs_default_opts(sfs_race_opts *opt);
+
+/* Table-1 features of A.  opt may be NULL (defaults; used for HYB width and
+   admissibility).  One fused device pass over row_ptr and col_idx + two small kernels.  Syncs.
+   Errors: INVALID_ARG (null/negative sizes), UNSUPPORTED (int32 overflow), INVALID_CSR, CUDA. */
+sfs_status sfs_features(const sfs_csr *A, const sfs_race_opts *opt, sfs_features_t *out, void *stream);
+
+/* Convert A into format f (step (ii) of P:L331) into a new library-owned handle *out.
+   Runs the feature pass internally (needed for widths / diagonals).  Syncs once (after features).
+   INADMISSIBLE for ELL / DIA past the fill guard (Q11).  For f = CSR with device input the handle
+   borrows A's arrays (the caller keeps them alive); with host input it owns device copies. */
+sfs_status sfs_convert(const sfs_csr *A, sfs_format f, const sfs_race_opts *opt, sfs_matrix *out, void *stream);
+
+/* y = A·x with A in format f (f must equal A's format, else INVALID_ARG).  x has ncols
+   entries, y has nrows entries, device pointers of A's dtype; y is fully overwritten.  Asynchronous:
+   1–2 kernel launches on `stream`, no synchronization. */
+sfs_status sfs_spmv(sfs_format f, sfs_matrix A, const void *x, void *y, void *stream);
+
+/* Label a batch of matrices: features of all n matrices (batched), then for each
+   matrix and each admissible format in opt->formats_mask: convert (event-timed), `warmup` untimed
+   SpMVs, `reps` timed SpMVs (CUDA events), free; label = argmin (Q14).  feats / labels are host
+   arrays of n entries.  A matrix-level error (e.g. INVALID_CSR) is reported in
+   labels[i].matrix_status and does not abort the batch; a format-level error (OOM) only marks
+   status[f].  Host-memory matrices are copied to the device inside the call and stay resident
+   until it returns (callers batch large corpora).  Syncs.  Returns SFS_OK unless an argument is
+   invalid or CUDA fails. */
+sfs_status sfs_label_corpus(const sfs_csr *mats, int64_t n, const sfs_race_opts *opt, sfs_features_t *feats,
+                            sfs_label_t *labels, void *stream);
+
+sfs_status sfs_matrix_free(sfs_matrix A); /* stream-ordered on the stream it was created on */
+sfs_status sfs_matrix_describe(sfs_matrix A, sfs_layout_t *out);
+
+/* Algorithmic bytes of one SpMV in format f for a matrix with features F and dtype (§8(a)
+   a9–a13: each format array read once, x read once, y written once; padding counted). */
+int64_t sfs_spmv_bytes(const sfs_features_t *F, sfs_format f, sfs_dtype dtype);
+
+const char *sfs_status_string(sfs_status s);
+const char *sfs_last_error(void);
+
+/* Allocator hook: both NULL restores the default pool.  alloc must return 256-byte aligned device
+   memory usable on `stream`; dealloc is called stream-ordered. */
+void sfs_set_allocator(void *(*alloc)(size_t bytes, void *stream), void (*dealloc)(void *p, void *stream));
+
+/* Number of kernels this library has launched in this process (graph replays count every node).
+   Lets benchmarks state how many of *our* kernels ran inside a timed region. */
+int64_t sfs_launch_count(void);
+
+/* Library version string. */
+const char *sfs_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

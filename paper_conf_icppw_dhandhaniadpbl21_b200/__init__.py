@@ -1,0 +1,304 @@
+"""B200-native sparse-format labelling path (Dhandhania et al., ICPP Workshops '21).
+
+Thin Python binding over the C ABI of ``include/sfs.h`` (``libsfs.so``, CUDA for sm_100a).  This
+module only marshals arguments: every step of the path (features, conversions, SpMV, the race)
+runs in the library's kernels.  PyTorch is used for device memory and streams only.  There is no
+CPU fallback: without the built library or a GPU every call raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass, field
+from typing import List, Optional, Sequence
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libsfs.so")
+
+CSR, COO, ELL, HYB, DIA = range(5)
+NFMT = 5
+FORMAT_NAMES = ["CSR", "COO", "ELL", "HYB", "DIA"]
+F32, F64 = 0, 1
+MEM_DEVICE, MEM_HOST = 0, 1
+
+OK, ERR_INVALID_ARG, ERR_INVALID_CSR, ERR_INADMISSIBLE, ERR_OOM, ERR_CUDA, ERR_UNSUPPORTED, ERR_NOT_RUN = (
+    0, -1, -2, -3, -4, -5, -6, -7)
+
+_I64, _I32, _U32, _D, _P = ctypes.c_int64, ctypes.c_int32, ctypes.c_uint32, ctypes.c_double, ctypes.c_void_p
+
+
+class SfsError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{msg} (status {status})")
+        self.status = status
+
+
+class CsrStruct(ctypes.Structure):
+    _fields_ = [("nrows", _I64), ("ncols", _I64), ("nnz", _I64), ("row_ptr", _P), ("col_idx", _P),
+                ("values", _P), ("dtype", _I32), ("mem", _I32), ("x", _P)]
+
+
+FEATURE_INT_FIELDS = ["nrows", "ncols", "nnz", "nnz_min", "nnz_max", "csr_max", "ell_size", "hyb_k",
+                      "hyb_ell_size", "hyb_coo", "hyb_ell_nnz", "diagonals", "dia_size"]
+FEATURE_FLOAT_FIELDS = ["nnz_frac", "nnz_mu", "nnz_sig", "max_mu", "mu_min", "sig_lower", "sig_higher",
+                        "hyb_ell_frac", "dia_frac", "ell_frac"]
+
+
+class FeaturesStruct(ctypes.Structure):
+    _fields_ = ([(f, _I64) for f in FEATURE_INT_FIELDS] + [(f, _D) for f in FEATURE_FLOAT_FIELDS]
+                + [("admissible_mask", _U32), ("csr_variant", _I32)])
+
+    def as_dict(self) -> dict:
+        d = {f: int(getattr(self, f)) for f in FEATURE_INT_FIELDS}
+        d.update({f: float(getattr(self, f)) for f in FEATURE_FLOAT_FIELDS})
+        d["admissible_mask"] = int(self.admissible_mask)
+        d["csr_variant"] = int(self.csr_variant)
+        return d
+
+
+class LayoutStruct(ctypes.Structure):
+    _fields_ = [("fmt", _I32), ("dtype", _I32), ("nrows", _I64), ("ncols", _I64), ("nnz", _I64), ("pitch", _I64),
+                ("width", _I64), ("ndiag", _I64), ("coo_nnz", _I64), ("ptr", _P * 6), ("bytes", _I64),
+                ("variant", _I32)]
+
+
+class RaceOpts(ctypes.Structure):
+    _fields_ = [("reps", _I32), ("warmup", _I32), ("formats_mask", _U32), ("cold", _I32), ("max_fill", _D),
+                ("fill_slack", _I64), ("hyb_rel_speed", _D), ("hyb_breakeven", _I64), ("csr_variant", _I32),
+                ("use_graphs", _I32)]
+
+
+class LabelStruct(ctypes.Structure):
+    _fields_ = [("label", _I32), ("admissible_mask", _U32), ("matrix_status", _I32), ("csr_variant", _I32),
+                ("t_spmv_us", ctypes.c_float * NFMT), ("t_convert_us", ctypes.c_float * NFMT),
+                ("status", _I32 * NFMT), ("bytes", _I64 * NFMT), ("t_features_us", ctypes.c_float)]
+
+    def as_dict(self) -> dict:
+        return {"label": int(self.label), "admissible_mask": int(self.admissible_mask),
+                "matrix_status": int(self.matrix_status), "csr_variant": int(self.csr_variant),
+                "t_spmv_us": list(self.t_spmv_us), "t_convert_us": list(self.t_convert_us),
+                "status": list(self.status), "bytes": list(self.bytes), "t_features_us": float(self.t_features_us)}
+
+
+_lib = None
+
+
+def lib():
+    """Load libsfs.so (fails loudly: there is no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: build it with __graft_entry__.build()")
+        L = ctypes.CDLL(LIB_PATH)
+        L.sfs_default_opts.argtypes = [ctypes.POINTER(RaceOpts)]
+        L.sfs_features.argtypes = [ctypes.POINTER(CsrStruct), ctypes.POINTER(RaceOpts), ctypes.POINTER(FeaturesStruct), _P]
+        L.sfs_convert.argtypes = [ctypes.POINTER(CsrStruct), _I32, ctypes.POINTER(RaceOpts), ctypes.POINTER(_P), _P]
+        L.sfs_spmv.argtypes = [_I32, _P, _P, _P, _P]
+        L.sfs_label_corpus.argtypes = [ctypes.POINTER(CsrStruct), _I64, ctypes.POINTER(RaceOpts),
+                                       ctypes.POINTER(FeaturesStruct), ctypes.POINTER(LabelStruct), _P]
+        L.sfs_matrix_free.argtypes = [_P]
+        L.sfs_matrix_describe.argtypes = [_P, ctypes.POINTER(LayoutStruct)]
+        L.sfs_spmv_bytes.argtypes = [ctypes.POINTER(FeaturesStruct), _I32, _I32]
+        L.sfs_spmv_bytes.restype = _I64
+        L.sfs_status_string.argtypes = [_I32]
+        L.sfs_status_string.restype = ctypes.c_char_p
+        L.sfs_last_error.restype = ctypes.c_char_p
+        L.sfs_launch_count.restype = _I64
+        L.sfs_version.restype = ctypes.c_char_p
+        for fn in ("sfs_features", "sfs_convert", "sfs_spmv", "sfs_label_corpus", "sfs_matrix_free",
+                   "sfs_matrix_describe"):
+            getattr(L, fn).restype = _I32
+        _lib = L
+    return _lib
+
+
+EXPORTED = ["sfs_features", "sfs_convert", "sfs_spmv", "sfs_label_corpus", "sfs_matrix_free",
+            "sfs_matrix_describe", "sfs_status_string", "sfs_last_error", "sfs_set_allocator",
+            "sfs_default_opts", "sfs_spmv_bytes", "sfs_launch_count", "sfs_version"]
+
+
+def _check(st: int, what: str):
+    if st != OK:
+        err = lib().sfs_last_error().decode(errors="replace")
+        raise SfsError(st, f"{what}: {lib().sfs_status_string(st).decode()} — {err}")
+
+
+def default_opts(**kw) -> RaceOpts:
+    o = RaceOpts()
+    lib().sfs_default_opts(ctypes.byref(o))
+    for k, v in kw.items():
+        if not hasattr(o, k):
+            raise AttributeError(k)
+        setattr(o, k, v)
+    return o
+
+
+def launch_count() -> int:
+    return int(lib().sfs_launch_count())
+
+
+def _stream_ptr(stream) -> Optional[int]:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream
+
+
+@dataclass
+class Csr:
+    """A CSR matrix held in torch tensors (device, or pinned host memory for the end-to-end path).
+    rp int32[m+1], col int32[nnz], val float32/float64[nnz]; x optional race input (ncols)."""
+    m: int
+    n: int
+    rp: "object"
+    col: "object"
+    val: "object"
+    x: "object" = None
+
+    @property
+    def nnz(self) -> int:
+        return int(self.col.numel())
+
+    @property
+    def dtype(self) -> int:
+        import torch
+        return F64 if self.val.dtype == torch.float64 else F32
+
+    def struct(self) -> CsrStruct:
+        import torch
+        for t in (self.rp, self.col):
+            assert t.dtype == torch.int32 and t.is_contiguous()
+        assert self.val.dtype in (torch.float32, torch.float64) and self.val.is_contiguous()
+        mem = MEM_DEVICE if self.rp.is_cuda else MEM_HOST
+        return CsrStruct(self.m, self.n, self.nnz, self.rp.data_ptr(), self.col.data_ptr(), self.val.data_ptr(),
+                         self.dtype, mem, self.x.data_ptr() if self.x is not None else None)
+
+    def nbytes(self) -> int:
+        return sum(t.numel() * t.element_size() for t in (self.rp, self.col, self.val))
+
+
+def csr_from_host(A, device="cuda", pin=False, with_x: Optional[int] = None) -> Csr:
+    """Move a host (numpy) CSR onto the device (or into pinned host memory)."""
+    import torch
+    if device == "host":
+        t = lambda a: torch.from_numpy(a).pin_memory() if pin else torch.from_numpy(a)
+    else:
+        t = lambda a: torch.from_numpy(a).to(device)
+    x = None
+    if with_x is not None:
+        import numpy as np
+        x = t(with_x) if isinstance(with_x, np.ndarray) else None
+    return Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), x)
+
+
+def features(A: Csr, opts: Optional[RaceOpts] = None, stream=None) -> dict:
+    """Table-1 features computed on the GPU (sfs_features)."""
+    f = FeaturesStruct()
+    s = A.struct()
+    _check(lib().sfs_features(ctypes.byref(s), ctypes.byref(opts) if opts else None, ctypes.byref(f),
+                              _stream_ptr(stream)), "sfs_features")
+    return f.as_dict()
+
+
+class Matrix:
+    """Library-owned converted matrix (sfs_matrix)."""
+
+    def __init__(self, handle, fmt, keepalive=None):
+        self.handle = handle
+        self.fmt = fmt
+        self._keep = keepalive
+
+    def layout(self) -> LayoutStruct:
+        L = LayoutStruct()
+        _check(lib().sfs_matrix_describe(self.handle, ctypes.byref(L)), "sfs_matrix_describe")
+        return L
+
+    def free(self):
+        if self.handle:
+            lib().sfs_matrix_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def convert(A: Csr, fmt: int, opts: Optional[RaceOpts] = None, stream=None) -> Matrix:
+    """CSR -> fmt on the GPU (sfs_convert)."""
+    h = ctypes.c_void_p()
+    s = A.struct()
+    _check(lib().sfs_convert(ctypes.byref(s), fmt, ctypes.byref(opts) if opts else None, ctypes.byref(h),
+                             _stream_ptr(stream)), f"sfs_convert({FORMAT_NAMES[fmt]})")
+    return Matrix(h.value, fmt, keepalive=A if fmt == CSR else None)
+
+
+def spmv(fmt: int, A: Matrix, x, y, stream=None):
+    """y = A x on the GPU (sfs_spmv); asynchronous on `stream`."""
+    _check(lib().sfs_spmv(fmt, A.handle, x.data_ptr(), y.data_ptr(), _stream_ptr(stream)), "sfs_spmv")
+    return y
+
+
+def label_corpus(mats: Sequence[Csr], opts: Optional[RaceOpts] = None, stream=None):
+    """Features + format race + labels for a batch (sfs_label_corpus).  Returns (features, labels)
+    as lists of dicts."""
+    n = len(mats)
+    arr = (CsrStruct * max(n, 1))(*[m.struct() for m in mats])
+    feats = (FeaturesStruct * max(n, 1))()
+    labs = (LabelStruct * max(n, 1))()
+    _check(lib().sfs_label_corpus(arr, n, ctypes.byref(opts) if opts else None, feats, labs, _stream_ptr(stream)),
+           "sfs_label_corpus")
+    return [feats[i].as_dict() for i in range(n)], [labs[i].as_dict() for i in range(n)]
+
+
+def spmv_bytes(feat: dict, fmt: int, dtype: int) -> int:
+    f = FeaturesStruct(*[feat[k] for k in FEATURE_INT_FIELDS], *[feat[k] for k in FEATURE_FLOAT_FIELDS],
+                       feat["admissible_mask"], feat.get("csr_variant", 0))
+    return int(lib().sfs_spmv_bytes(ctypes.byref(f), fmt, dtype))
+
+
+def decode(M: Matrix):
+    """Copy a converted matrix's arrays to the host (numpy), following the documented layout of
+    sfs_layout_t.  Test / inspection helper only (no arithmetic)."""
+    import numpy as np
+    import torch
+    L = M.layout()
+    vt = torch.float64 if L.dtype == F64 else torch.float32
+    ne = int
+
+    def fetch(ptr, n, dtype):
+        np_t = {torch.int32: np.int32, torch.float32: np.float32, torch.float64: np.float64}[dtype]
+        if n == 0:
+            return np.zeros(0, dtype=np_t)
+        torch.cuda.synchronize()
+        return torch.as_tensor(_DevView(ptr, n, np.dtype(np_t).str), device="cuda").cpu().numpy().copy()
+
+    P, K, m = L.pitch, L.width, L.nrows
+    r = {"pitch": P, "width": K, "ndiag": L.ndiag, "coo_nnz": L.coo_nnz, "variant": L.variant, "bytes": L.bytes}
+    if L.fmt == CSR:
+        r.update(rp=fetch(L.ptr[0], m + 1, torch.int32), col=fetch(L.ptr[1], ne(L.nnz), torch.int32),
+                 val=fetch(L.ptr[2], ne(L.nnz), vt))
+    elif L.fmt == COO:
+        r.update(row=fetch(L.ptr[0], ne(L.nnz), torch.int32), col=fetch(L.ptr[1], ne(L.nnz), torch.int32),
+                 val=fetch(L.ptr[2], ne(L.nnz), vt))
+    elif L.fmt in (ELL, HYB):
+        r.update(ecol=fetch(L.ptr[0], K * P, torch.int32).reshape(K, P) if K else np.zeros((0, P), np.int32),
+                 eval=fetch(L.ptr[1], K * P, vt).reshape(K, P) if K else np.zeros((0, P)))
+        if L.fmt == HYB:
+            c = ne(L.coo_nnz)
+            r.update(crow=fetch(L.ptr[2], c, torch.int32), ccol=fetch(L.ptr[3], c, torch.int32),
+                     cval=fetch(L.ptr[4], c, vt))
+    elif L.fmt == DIA:
+        nd = ne(L.ndiag)
+        r.update(offs=fetch(L.ptr[0], nd, torch.int32),
+                 dval=fetch(L.ptr[1], nd * P, vt).reshape(nd, P) if nd else np.zeros((0, P)))
+    return r
+
+
+class _DevView:
+    """Zero-copy view of library-owned device memory (__cuda_array_interface__) for decode()."""
+
+    def __init__(self, ptr: int, n: int, typestr: str):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, True), "version": 3,
+                                         "strides": None}

@@ -1,0 +1,115 @@
+// internal.h — host-side internals of libsfs (not part of the ABI).
+#pragma once
+#include <cuda_runtime.h>
+#include <stddef.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <string>
+
+#include "sfs.h"
+#include "shape.h"
+
+namespace sfs {
+
+// ---------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+#define SFS_CUDA_TRY(expr)                                                                          \
+  do {                                                                                              \
+    cudaError_t _e = (expr);                                                                        \
+    if (_e != cudaSuccess) {                                                                        \
+      ::sfs::set_error(std::string(#expr) + ": " + cudaGetErrorString(_e) + " @" + __FILE__ + ":" + \
+                       std::to_string(__LINE__));                                                   \
+      return _e == cudaErrorMemoryAllocation ? SFS_ERR_OOM : SFS_ERR_CUDA;                          \
+    }                                                                                               \
+  } while (0)
+
+// ---------------------------------------------------------------- memory
+void* dalloc(size_t bytes, cudaStream_t s);  // nullptr on failure
+void dfree(void* p, cudaStream_t s);
+
+// kernels launched by this library (sfs_launch_count)
+extern std::atomic<int64_t> g_launches;
+inline void count_launch(int64_t n = 1) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+
+// ---------------------------------------------------------------- feature pass (features.cu)
+constexpr int kHistCap = 4096;  // exact row-length histogram bins [0, 4095]; bin 4096 = ">= 4096"
+
+struct DevAggr {                // zeroed by memset; every field updated with atomics
+  unsigned long long flags;     // validation error bits (Q16)
+  unsigned long long min_inv;   // max over rows of (INT32_MAX - len)
+  unsigned long long max_len;
+  unsigned long long S2, cL, s1L, s2L, cH, s1H, s2H;
+  unsigned long long ndiag;
+  unsigned long long big_cnt, big_sum;  // rows with len >= kHistCap
+  long long hyb_k;                      // -1: order statistic beyond the histogram, host refines
+  long long hyb_coo;
+  long long pad[2];
+};
+
+enum : unsigned long long {
+  FLAG_RP0 = 1, FLAG_RP_DECREASE = 2, FLAG_RP_END = 4, FLAG_COL_RANGE = 8, FLAG_COL_ORDER = 16
+};
+
+struct FeatWork {
+  void* base = nullptr;
+  size_t bytes = 0;
+  DevAggr* aggr = nullptr;
+  unsigned* hist = nullptr;    // kHistCap + 1
+  unsigned* bitmap = nullptr;  // words
+  long long words = 0;         // ceil((m + n - 1) / 32)
+};
+
+size_t feat_work_bytes(long long m, long long n);
+void feat_work_bind(FeatWork& w, void* base, long long m, long long n);
+// memset + row stats + nnz pass + diag count + HYB select (4 kernels + 1 memset)
+cudaError_t launch_features(const int* rp, const int* col, long long m, long long n, long long z, long long rmax,
+                            const FeatWork& w, cudaStream_t s);
+// refine pass of the HYB order statistic: histogram of lengths in [lo, hi] with bin width wdt
+cudaError_t launch_len_hist_range(const int* rp, long long m, long long lo, long long hi, long long wdt,
+                                  unsigned* hist, cudaStream_t s);
+cudaError_t launch_hyb_coo(const int* rp, long long m, long long K, long long* out, cudaStream_t s);
+
+// ---------------------------------------------------------------- scans (scan.cu)
+// exclusive scan of transformed per-row values; out has m+1 entries (out[m] = total)
+size_t scan_work_bytes(long long m);
+cudaError_t launch_overflow_scan(const int* rp, long long m, int K, int* out, void* work, cudaStream_t s);
+cudaError_t launch_popc_scan(const unsigned* words, long long nw, int* out, void* work, cudaStream_t s);
+
+// ---------------------------------------------------------------- conversions (convert.cu)
+cudaError_t launch_csr2coo(int dtype, const int* rp, const int* col, const void* val, long long m, long long z,
+                           int* orow, int* ocol, void* oval, cudaStream_t s);
+// ELL slab (and the ELL part of HYB): width K, pitch P
+cudaError_t launch_csr2ell(int dtype, const int* rp, const int* col, const void* val, long long m, long long P,
+                           int K, int* ecol, void* eval, cudaStream_t s);
+// COO part of HYB: entries j >= K of each row, placed at ovf[r] + j - K
+cudaError_t launch_hyb_coo_part(int dtype, const int* rp, const int* col, const void* val, long long m,
+                                long long z, int K, const int* ovf, int* crow, int* ccol, void* cval,
+                                cudaStream_t s);
+cudaError_t launch_dia_offsets(const unsigned* bitmap, long long nw, const int* wprefix, long long m, int* offs,
+                               cudaStream_t s);
+cudaError_t launch_csr2dia(int dtype, const int* rp, const int* col, const void* val, long long m,
+                           long long P, const unsigned* bitmap, const int* wprefix, void* dval, cudaStream_t s);
+
+// ---------------------------------------------------------------- SpMV (spmv.cu)
+struct Matrix;
+int spmv_kernels_per_call(const Matrix* A);
+cudaError_t launch_spmv(const Matrix* A, const void* x, void* y, cudaStream_t s);
+size_t csr_merge_work_bytes(long long m, long long z, int dtype);
+int csr_vector_tpv(long long m, long long z);
+cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
+
+// ---------------------------------------------------------------- matrix handle
+struct Matrix {
+  int fmt = 0, dtype = 0;
+  long long m = 0, n = 0, nnz = 0, pitch = 0, width = 0, ndiag = 0, coo_nnz = 0;
+  const void* ptr[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+  void* owned[8] = {nullptr};  // buffers to free
+  int n_owned = 0;
+  long long bytes = 0;
+  int variant = 0;             // CSR: 0 vector, 1 merge
+  void* work = nullptr;        // CSR merge carries
+  cudaStream_t stream = nullptr;
+};
+
+}  // namespace sfs

@@ -1,0 +1,52 @@
+"""GPU parity at BASELINE.json's full sizes (configs[0], [2], [3] and a slice of configs[1]),
+through the same C-ABI calls the bench times."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+import sfsgen
+from gpu_util import assert_features_equal, check_conversion, check_spmv, to_dev
+
+pytestmark = pytest.mark.gpu
+
+
+def _full_check(A, formats=range(5), conv=True, ctx=""):
+    fo = oracle.features(A.m, A.n, A.rp, A.col)
+    dA = to_dev(A)
+    assert_features_equal(sfs.features(dA), fo, ctx)
+    x = sfsgen.vector(2024, A.n, A.dtype)
+    for fmt in formats:
+        if not (fo["admissible_mask"] >> fmt) & 1:
+            continue
+        M = sfs.convert(dA, fmt)
+        if conv:
+            check_conversion(A, fmt, M, fo)
+        check_spmv(A, fmt, M, x, A.dtype, ctx=ctx)
+        M.free()
+    return fo
+
+
+def test_config0_laplace_64_fp64():
+    A = sfsgen.laplace2d(64)
+    fo = _full_check(A, ctx="configs[0]")
+    assert fo["admissible_mask"] == 31
+
+
+def test_config2_rmat_22_fp32():
+    A = sfsgen.rmat(22, seed=1)
+    fo = _full_check(A, formats=(sfs.CSR, sfs.COO, sfs.HYB), conv=True, ctx="configs[2]")
+    assert not (fo["admissible_mask"] >> sfs.ELL) & 1 and not (fo["admissible_mask"] >> sfs.DIA) & 1
+    assert fo["nnz"] > 60_000_000 and fo["nnz_max"] > 50_000
+
+
+def test_config3_stencil3d27_128_fp64():
+    A = sfsgen.stencil3d27(128)
+    fo = _full_check(A, ctx="configs[3]")
+    assert (fo["nnz"], fo["diagonals"], fo["hyb_k"]) == (55742968, 27, 27)
+
+
+@pytest.mark.parametrize("i", [0, 1, 2, 3, 4, 5, 6, 7])
+def test_config1_corpus_slice(i):
+    A = sfsgen.generate(sfsgen.corpus_spec(200, i))
+    _full_check(A, conv=(A.nnz < 20_000_000), ctx=f"corpus200[{i}]")

@@ -1,0 +1,233 @@
+"""GPU parity: the CUDA path (through the C ABI) against the CPU oracle on the same seeded inputs.
+
+Bars (BASELINE.json north_star): features and conversions bit-exact; SpMV per row
+|y - y_ref| <= tol * (|A||x|)_r with tol 1e-12 (fp64) / 1e-5 (fp32), rows with |A||x| = 0 exactly 0.
+"""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+import sfsgen
+from gpu_util import assert_features_equal, check_conversion, check_spmv, to_dev
+from helpers import golden, random_csr
+
+pytestmark = pytest.mark.gpu
+
+
+def _cases():
+    rng = np.random.default_rng(1234)
+    cases = {
+        "tiny4x4": sfsgen.from_dense(np.array(golden("tiny4x4.json")["A"], float)),
+        "1x1": sfsgen.from_dense(np.array([[2.5]])),
+        "empty": sfsgen.CSR(7, 5, np.zeros(8, np.int32), np.zeros(0, np.int32), np.zeros(0)),
+        "laplace64": sfsgen.laplace2d(64),
+        "rand_ragged": random_csr(rng, 3001, 2777, 0.004, empty_rows=0.3, dense_rows=2),
+        "rand_zeros": random_csr(rng, 500, 700, 0.02, explicit_zero=0.2),
+        "band": sfsgen.generate(sfsgen.make_spec(sfsgen.BAND, seed=3, m=20011, ia=9, pa=0.7)),
+        "blockdiag32": sfsgen.generate(sfsgen.make_spec(sfsgen.BLOCKDIAG, seed=4, m=9001, ia=37, pa=0.8,
+                                                         dtype=sfsgen.F32)),
+        "uniform": sfsgen.generate(sfsgen.make_spec(sfsgen.UNIFORM, seed=5, m=12000, n=9000, pa=17.0)),
+        "powerlaw32": sfsgen.generate(sfsgen.make_spec(sfsgen.POWERLAW, seed=6, m=30000, pa=2.15, dtype=sfsgen.F32)),
+        "rmat14": sfsgen.rmat(14, seed=7),
+        "st3d27_20": sfsgen.generate(sfsgen.make_spec(sfsgen.ST3D27, ia=20)),
+        "st3d7_32f": sfsgen.generate(sfsgen.make_spec(sfsgen.ST3D7, ia=33, dtype=sfsgen.F32)),
+    }
+    return cases
+
+
+CASES = None
+
+
+def cases():
+    global CASES
+    if CASES is None:
+        CASES = _cases()
+    return CASES
+
+
+NAMES = ["tiny4x4", "1x1", "empty", "laplace64", "rand_ragged", "rand_zeros", "band", "blockdiag32", "uniform",
+         "powerlaw32", "rmat14", "st3d27_20", "st3d7_32f"]
+
+
+@pytest.mark.parametrize("name", NAMES)
+def test_features_bit_exact(name):
+    A = cases()[name]
+    fg = sfs.features(to_dev(A))
+    fo = oracle.features(A.m, A.n, A.rp, A.col)
+    assert_features_equal(fg, fo, name)
+
+
+@pytest.mark.parametrize("name", NAMES)
+def test_conversions_bit_exact(name):
+    A = cases()[name]
+    fo = oracle.features(A.m, A.n, A.rp, A.col)
+    dA = to_dev(A)
+    for fmt in range(5):
+        if not (fo["admissible_mask"] >> fmt) & 1:
+            with pytest.raises(sfs.SfsError) as ei:
+                sfs.convert(dA, fmt)
+            assert ei.value.status == sfs.ERR_INADMISSIBLE
+            continue
+        M = sfs.convert(dA, fmt)
+        check_conversion(A, fmt, M, fo)
+        M.free()
+
+
+@pytest.mark.parametrize("name", NAMES)
+@pytest.mark.parametrize("variant", [0, 1])
+def test_spmv_tolerance(name, variant):
+    A = cases()[name]
+    fo = oracle.features(A.m, A.n, A.rp, A.col)
+    x = sfsgen.vector(99, A.n, A.dtype)
+    dA = to_dev(A)
+    opts = sfs.default_opts(csr_variant=variant)
+    for fmt in range(5):
+        if not (fo["admissible_mask"] >> fmt) & 1:
+            continue
+        if fmt != sfs.CSR and variant == 1:
+            continue
+        M = sfs.convert(dA, fmt, opts)
+        check_spmv(A, fmt, M, x, A.dtype, ctx=f"{name}/v{variant}")
+        M.free()
+
+
+@pytest.mark.parametrize("dtype", [sfsgen.F64, sfsgen.F32])
+@pytest.mark.parametrize("cls,N,pts", [(sfsgen.ST2D5, 64, 5), (sfsgen.ST3D27, 24, 27)])
+def test_spmv_x_ones_bitwise(dtype, cls, N, pts):
+    """x = 1 on a stencil: every partial sum is a small integer, so every format in both precisions
+    must give y = points - len exactly (SURVEY §8(c) exact special case)."""
+    import torch
+    A = sfsgen.generate(sfsgen.make_spec(cls, ia=N, dtype=dtype))
+    expect = (pts - np.diff(A.rp)).astype(np.float64)
+    dA = to_dev(A)
+    tdt = torch.float64 if dtype == sfsgen.F64 else torch.float32
+    x = torch.ones(A.n, dtype=tdt, device="cuda")
+    for variant in (0, 1):
+        for fmt in range(5):
+            if variant == 1 and fmt != sfs.CSR:
+                continue
+            M = sfs.convert(dA, fmt, sfs.default_opts(csr_variant=variant))
+            y = torch.empty(A.m, dtype=tdt, device="cuda")
+            sfs.spmv(fmt, M, x, y)
+            assert (y.cpu().numpy().astype(np.float64) == expect).all(), sfs.FORMAT_NAMES[fmt]
+
+
+def test_spmv_unit_vector_bitwise():
+    import torch
+    A = cases()["rand_ragged"]
+    dense_col = np.zeros(A.m)
+    j = 17
+    for r in range(A.m):
+        for k in range(A.rp[r], A.rp[r + 1]):
+            if A.col[k] == j:
+                dense_col[r] = A.val[k]
+    dA = to_dev(A)
+    e = torch.zeros(A.n, dtype=torch.float64, device="cuda")
+    e[j] = 1.0
+    fo = oracle.features(A.m, A.n, A.rp, A.col)
+    for fmt in range(5):
+        if (fo["admissible_mask"] >> fmt) & 1:
+            M = sfs.convert(dA, fmt)
+            y = torch.empty(A.m, dtype=torch.float64, device="cuda")
+            sfs.spmv(fmt, M, e, y)
+            assert (y.cpu().numpy() == dense_col).all()
+
+
+def test_hyb_order_statistic_refine_path():
+    """HYB width beyond the exact histogram (>= 4096 rows of length >= 4096) -> host refinement."""
+    m, n = 4500, 9700
+    lens = 4096 + (np.arange(m) * 7919) % 700
+    rp = np.concatenate([[0], np.cumsum(lens)]).astype(np.int32)
+    col = np.concatenate([np.arange(L) * 2 + (r % 2) for r, L in enumerate(lens)]).astype(np.int32)
+    A = sfsgen.CSR(m, n, rp, col, np.ones(len(col)))
+    fg = sfs.features(to_dev(A))
+    fo = oracle.features(m, n, rp, col)
+    assert fo["hyb_k"] >= 4096
+    assert_features_equal(fg, fo, "refine")
+
+
+def test_errors():
+    import torch
+    A = cases()["laplace64"]
+    bad = sfsgen.CSR(A.m, A.n, A.rp.copy(), A.col.copy(), A.val)
+    bad.col[10], bad.col[11] = bad.col[11], bad.col[10]  # not increasing
+    with pytest.raises(sfs.SfsError) as ei:
+        sfs.features(to_dev(bad))
+    assert ei.value.status == sfs.ERR_INVALID_CSR
+    bad2 = sfsgen.CSR(A.m, A.n, A.rp.copy(), A.col.copy(), A.val)
+    bad2.rp[100] = bad2.rp[101] + 1  # decreasing row_ptr
+    with pytest.raises(sfs.SfsError) as ei:
+        sfs.features(to_dev(bad2))
+    assert ei.value.status == sfs.ERR_INVALID_CSR
+    bad3 = sfsgen.CSR(A.m, 50, A.rp, A.col, A.val)  # column out of range
+    with pytest.raises(sfs.SfsError) as ei:
+        sfs.features(to_dev(bad3))
+    assert ei.value.status == sfs.ERR_INVALID_CSR
+    M = sfs.convert(to_dev(A), sfs.COO)
+    x = torch.ones(A.n, dtype=torch.float64, device="cuda")
+    y = torch.empty(A.m, dtype=torch.float64, device="cuda")
+    with pytest.raises(sfs.SfsError) as ei:
+        sfs.spmv(sfs.CSR, M, x, y)
+    assert ei.value.status == sfs.ERR_INVALID_ARG
+    anti = sfsgen.CSR(3000, 3000, np.arange(3001, dtype=np.int32), (2999 - np.arange(3000)).astype(np.int32),
+                      np.ones(3000))
+    with pytest.raises(sfs.SfsError) as ei:
+        sfs.convert(to_dev(anti), sfs.DIA, sfs.default_opts(fill_slack=0))
+    assert ei.value.status == sfs.ERR_INADMISSIBLE
+
+
+def test_host_memory_input_matches_device():
+    """The end-to-end path (host CSR, copies inside the call) computes the same features."""
+    import torch
+    A = cases()["uniform"]
+    host = sfs.Csr(A.m, A.n, torch.from_numpy(A.rp).pin_memory(), torch.from_numpy(A.col).pin_memory(),
+                   torch.from_numpy(A.val).pin_memory())
+    assert_features_equal(sfs.features(host), oracle.features(A.m, A.n, A.rp, A.col), "host")
+    M = sfs.convert(host, sfs.HYB)
+    check_conversion(A, sfs.HYB, M, oracle.features(A.m, A.n, A.rp, A.col))
+
+
+def test_label_corpus_small():
+    names = ["laplace64", "band", "blockdiag32", "uniform", "powerlaw32", "rmat14", "empty", "tiny4x4"]
+    mats = [to_dev(cases()[k]) for k in names]
+    opts = sfs.default_opts(reps=20, warmup=2)
+    feats, labs = sfs.label_corpus(mats, opts)
+    for k, f, L in zip(names, feats, labs):
+        A = cases()[k]
+        fo = oracle.features(A.m, A.n, A.rp, A.col)
+        assert_features_equal(f, fo, k)
+        assert L["matrix_status"] == 0 and L["admissible_mask"] == fo["admissible_mask"]
+        ran = [i for i in range(5) if L["status"][i] == 0]
+        assert ran == [i for i in range(5) if (fo["admissible_mask"] >> i) & 1]
+        t = np.array(L["t_spmv_us"], dtype=np.float64)
+        assert all(t[i] > 0 for i in ran)
+        # decision rule (Q14) reproduced by the oracle from the measured times
+        assert L["label"] == oracle.label(t, sum(1 << i for i in ran))
+        for i in range(5):
+            assert L["bytes"][i] == sfs.spmv_bytes(f, i, A.dtype)
+        assert L["t_convert_us"][0] == 0 and all(L["t_convert_us"][i] > 0 for i in ran if i)
+    # masks: the paper's four formats only
+    feats2, labs2 = sfs.label_corpus(mats[:2], sfs.default_opts(reps=5, warmup=1, formats_mask=0x0F))
+    assert all(L["status"][4] == sfs.ERR_NOT_RUN and L["label"] != 4 for L in labs2)
+
+
+def test_label_corpus_invalid_matrix_does_not_abort():
+    A = cases()["laplace64"]
+    bad = sfsgen.CSR(A.m, A.n, A.rp.copy(), A.col.copy(), A.val)
+    bad.col[5] = bad.col[4]
+    feats, labs = sfs.label_corpus([to_dev(bad), to_dev(A)], sfs.default_opts(reps=3, warmup=1))
+    assert labs[0]["matrix_status"] == sfs.ERR_INVALID_CSR and labs[0]["label"] == -1
+    assert labs[1]["matrix_status"] == 0 and labs[1]["label"] >= 0
+
+
+def test_launch_count_increases():
+    import torch
+    A = cases()["band"]
+    M = sfs.convert(to_dev(A), sfs.COO)
+    x = torch.ones(A.n, dtype=torch.float64, device="cuda")
+    y = torch.empty(A.m, dtype=torch.float64, device="cuda")
+    c0 = sfs.launch_count()
+    for _ in range(3):
+        sfs.spmv(sfs.COO, M, x, y)
+    assert sfs.launch_count() - c0 == 6  # memset + kernel per COO SpMV
