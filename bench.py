@@ -1,0 +1,368 @@
+#!/usr/bin/env python
+"""bench.py — matrices labelled per second on the BASELINE configs[1] corpus (the headline metric).
+
+One step = the whole hot path (SURVEY §8(a) a1–a15) over one batch: for every matrix of the rank's
+corpus-200 (configs[1]: banded / uniform random / block-diagonal / power-law, 10K–1M rows, fp32 and
+fp64 values) the Table-1 feature pass, every admissible conversion, the device-timed format race
+(5 warm-up + 100 timed SpMVs per format) and the label; at N > 1 the labels/features are
+gathered over NCCL.  Inputs are resident in HBM when the timed region starts (`value`); `e2e`
+repeats the step through the same C-ABI call with pinned HOST buffers (H2D inside the call).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+`--impl reference` times the CPU oracle (the only reference that exists: the paper ships no code)
+on the box's host cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "matrices labelled/s (features + all-format conversion + 100-rep SpMV race + label), corpus-200"
+UNIT = "matrices/s"
+DAGGR_BYTES = 136  # device aggregate record copied back per matrix (internal.h DevAggr)
+LABEL_BYTES = 4 * 4 + 5 * 4 * 3 + 5 * 8 + 4  # sfs_label_t
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=3)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--corpus", type=int, default=200, help="matrices per rank (configs[1]: 200)")
+    p.add_argument("--reps", type=int, default=100)
+    p.add_argument("--race-warmup", type=int, default=5)
+    p.add_argument("--e2e-steps", type=int, default=2)
+    p.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--out", default=None, help="also append the JSON line to this file")
+    return p.parse_args()
+
+
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def corpus_ids(rank, per_rank):
+    """Weak scaling: rank r labels matrices [r*per_rank, (r+1)*per_rank) of the configs[1] recipe."""
+    return list(range(rank * per_rank, (rank + 1) * per_rank))
+
+
+def generate_host(ids):
+    import sfsgen
+    mats = []
+    for i in ids:
+        A = sfsgen.generate(sfsgen.corpus_spec(200, i))
+        x = sfsgen.vector(sfsgen.corpus_spec(200, i).seed, A.n, A.dtype)
+        mats.append((i, A, x))
+    return mats
+
+
+# ------------------------------------------------------------------ clocks (nvidia-smi during the timed region)
+class ClockSampler:
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "200"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [v.strip() for v in ln.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ------------------------------------------------------------------ CPU oracle (cpu_baseline / reference arm)
+def oracle_sample(host_mats, budget_s, threads, reps=100):
+    """Run the oracle's whole labelling pass on matrices in corpus order, `threads` at a time, until
+    `budget_s` of wall time is spent.  Returns (matrices/s, completed, cores, wall)."""
+    import oracle
+    from concurrent.futures import ThreadPoolExecutor, FIRST_COMPLETED, wait
+
+    t0 = time.perf_counter()
+    done = 0
+    nnz = 0
+    it = iter(host_mats)
+    futs = set()
+
+    def job(item):
+        _, A, x = item
+        oracle.label_matrix(A.m, A.n, A.rp, A.col, A.val.astype(np.float64), x.astype(np.float64), reps=reps)
+        return A.nnz
+
+    with ThreadPoolExecutor(max_workers=threads) as ex:
+        for _ in range(threads):
+            nxt = next(it, None)
+            if nxt is None:
+                break
+            futs.add(ex.submit(job, nxt))
+        while futs:
+            fin, futs = wait(futs, return_when=FIRST_COMPLETED)
+            for f in fin:
+                nnz += f.result()
+                done += 1
+            if time.perf_counter() - t0 < budget_s:
+                for _ in range(len(fin)):
+                    nxt = next(it, None)
+                    if nxt is not None:
+                        futs.add(ex.submit(job, nxt))
+    wall = time.perf_counter() - t0
+    return done / wall, done, threads, wall, nnz
+
+
+def run_reference(args):
+    rank, world, _ = dist_env()
+    if rank != 0:
+        return 0
+    host = generate_host(corpus_ids(0, args.corpus))
+    threads = os.cpu_count() or 1
+    budget = max(5.0, min(args.cpu_budget, 20.0))
+    for _ in range(args.warmup):
+        oracle_sample(host, budget / 4, threads, reps=args.reps)
+    vals, walls, done = [], [], []
+    for _ in range(args.steps):
+        v, d, c, w, nnz = oracle_sample(host, budget, threads, reps=args.reps)
+        vals.append(v)
+        walls.append(w)
+        done.append(d)
+    value = statistics.median(vals)
+    sample = (f"first {min(done)}-{max(done)} matrices (corpus order) of corpus-200 per step, oracle labelling "
+              f"pass (features + conversions + {args.reps} reps/format + argmin), {threads} threads, ~{budget:.0f} s/step")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * statistics.median(walls),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": "corpus-200 (BASELINE configs[1])", "matrices_per_rank": args.corpus},
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ------------------------------------------------------------------ our arm
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+
+    rank, world, local = dist_env()
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    stream = torch.cuda.current_stream()
+
+    host = generate_host(corpus_ids(rank, args.corpus))
+    t = lambda a: torch.from_numpy(a).to(dev)
+    mats = [sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), t(x)) for _, A, x in host]
+    pin = lambda a: torch.from_numpy(a).pin_memory()
+    hmats = [sfs.Csr(A.m, A.n, pin(A.rp), pin(A.col), pin(A.val), pin(x)) for _, A, x in host]
+    torch.cuda.synchronize()
+    opts = sfs.default_opts(reps=args.reps, warmup=args.race_warmup)
+    n = len(mats)
+    gather_buf = torch.zeros(n * 8, dtype=torch.float64, device=dev)
+    all_buf = torch.zeros(world * n * 8, dtype=torch.float64, device=dev)
+
+    def step(batch):
+        feats, labs = sfs.label_corpus(batch, opts)
+        if world > 1:  # a15: gather labels + timing summary to every rank (results, ~64 B / matrix)
+            rows = [[L["label"]] + L["t_spmv_us"] + [L["t_features_us"], L["matrix_status"]] for L in labs]
+            gather_buf.copy_(torch.tensor(rows, dtype=torch.float64).reshape(-1))
+            dist.all_gather_into_tensor(all_buf, gather_buf)
+        return feats, labs
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def maxr(v):
+        if world == 1:
+            return v
+        tt = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
+
+    def sumr(v):
+        if world == 1:
+            return v
+        tt = torch.tensor([v], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.SUM)
+        return float(tt.item())
+
+    for _ in range(args.warmup):
+        step(mats)
+    # ---- timed region: K steps, inputs resident in HBM
+    clocks = ClockSampler(local)
+    clocks.start()
+    barrier()
+    l0 = sfs.launch_count()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    results = []
+    for _ in range(args.steps):
+        results.append(step(mats))
+    e1.record(stream)
+    barrier()
+    clk = clocks.stop()
+    launches = sfs.launch_count() - l0
+    t_dev = e0.elapsed_time(e1) / 1000.0
+    t_max = maxr(t_dev)
+    total_mats = world * n * args.steps
+    value = total_mats / t_max
+    launches_all = int(sumr(float(launches)))
+
+    # ---- e2e: same call with pinned host inputs (H2D inside the call), result D2H inside
+    barrier()
+    e2 = torch.cuda.Event(enable_timing=True)
+    e3 = torch.cuda.Event(enable_timing=True)
+    e2.record(stream)
+    for _ in range(args.e2e_steps):
+        step(hmats)
+    e3.record(stream)
+    barrier()
+    t_e2e = maxr(e2.elapsed_time(e3) / 1000.0)
+    h2d = sum(m.nbytes() + m.x.numel() * m.x.element_size() for m in hmats)
+    e2e = {"value": world * n * args.e2e_steps / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d,
+           "d2h_bytes_per_step": n * DAGGR_BYTES}
+
+    # ---- roofline of the dominant kernel (from the race's own CUDA events, inside the timed region)
+    feats, labs = results[-1]
+    per_fmt = {}
+    for f in range(sfs.NFMT):
+        tt = sum(L["t_spmv_us"][f] for L in labs if L["status"][f] == 0) * args.reps
+        bb = sum(L["bytes"][f] for L in labs if L["status"][f] == 0) * args.reps
+        big = [(L["bytes"][f], L["t_spmv_us"][f]) for L in labs if L["status"][f] == 0 and L["bytes"][f] > 256e6]
+        per_fmt[sfs.FORMAT_NAMES[f]] = {
+            "matrices": sum(1 for L in labs if L["status"][f] == 0),
+            "spmv_time_s": tt / 1e6, "gbs": (bb / (tt / 1e6) / 1e9) if tt else None,
+            "gbs_footprint_gt_2xL2": (sum(b for b, _ in big) / (sum(t for _, t in big) / 1e6) / 1e9) if big else None,
+            "labels": sum(1 for L in labs if L["label"] == f),
+            "convert_over_csr_spmv": (statistics.median(
+                [L["t_convert_us"][f] / L["t_spmv_us"][0] for L in labs
+                 if L["status"][f] == 0 and L["status"][0] == 0 and L["t_spmv_us"][0] > 0]) if f else 0.0),
+        }
+    dom = max(per_fmt, key=lambda k: per_fmt[k]["spmv_time_s"])
+    peaks = {}
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as fh:
+            peaks = json.load(fh)
+    except Exception:
+        pass
+    peak = peaks.get("hbm_gbs")
+    peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
+    if not peak:
+        peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
+    traffic = None
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
+            traffic = json.load(fh).get(dom)
+    except Exception:
+        pass
+    achieved = per_fmt[dom]["gbs"]
+    step_time = t_dev / args.steps
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak if achieved else None, "traffic": traffic,
+                "kernel": f"SpMV {dom} ({'k_spmv_csr_vector / k_spmv_csr_merge' if dom == 'CSR' else 'k_spmv_' + dom.lower()})",
+                "peak_source": peak_src,
+                "share_of_step": per_fmt[dom]["spmv_time_s"] / step_time,
+                "note": "achieved = sum over matrices of algorithmic bytes (SURVEY 8(a) a9-a13) x reps / sum of "
+                        "event-timed race time; hot back-to-back reps (P:L217), so matrices that fit in L2 count at "
+                        "L2 speed; gbs_footprint_gt_2xL2 in per_format restricts to footprints > 256 MB"}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        threads = os.cpu_count() or 1
+        v, d, c, w, nnz = oracle_sample(host, args.cpu_budget, threads, reps=args.reps)
+        cpu = {"value": v, "unit": UNIT, "cores": c, "kind": "oracle",
+               "sample": f"first {d} matrices of this rank's corpus-200 in corpus order ({nnz} nnz), oracle labelling "
+                         f"pass (features + conversions + {args.reps} SpMV reps/format + argmin, as the GPU step), "
+                         f"{c} threads, {w:.1f} s"}
+
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": 1000 * t_max / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "config": {"workload": "corpus-200 (BASELINE configs[1]): banded/uniform/block-diagonal/power-law, "
+                                       "10K-1M rows, values fp32 and fp64 (half each), SpMV accumulates in fp64",
+                           "matrices_per_rank": n, "nnz_per_rank": int(sum(m.nnz for m in mats)),
+                           "reps": args.reps, "race_warmup": args.race_warmup,
+                           "parallelism": f"corpus sharded over {world} GPU(s), no data-path collective",
+                           "l2": "inputs larger than L2 (corpus >> 126 MB per step); in-race reps back-to-back (P:L217)"},
+                "e2e": e2e, "gpu_launches": launches_all, "clocks": clk, "roofline": roofline,
+                "cpu_baseline": cpu, "per_format": per_fmt,
+                "label_histogram": {k: v["labels"] for k, v in per_fmt.items()}}
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.out:
+            with open(args.out, "a") as fh:
+                fh.write(s + "\n")
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return run_reference(args)
+    return run_ours(args)
+
+
+if __name__ == "__main__":
+    sys.exit(main())

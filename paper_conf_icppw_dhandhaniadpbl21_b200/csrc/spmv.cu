@@ -361,8 +361,12 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       const int* col = (const int*)A->ptr[1];
       const T* val = (const T*)A->ptr[2];
       if (A->variant == 0) {
-        const int blocks = kCsrWarps * 32 / 256;
-        switch (csr_vector_tpv(m, z)) {
+        // kCsrWarps warps grid-stride over rows (the mapping the csr_max feature describes, Q4); a
+        // matrix covered in one pass gets only the warps that own rows (same row -> warp mapping).
+        const int tpv = csr_vector_tpv(m, z);
+        const long long warps_needed = ceil_div(m, 32 / tpv);
+        const int blocks = (int)ceil_div(warps_needed < kCsrWarps ? warps_needed : kCsrWarps, 256 / 32);
+        switch (tpv) {
           case 2: k_spmv_csr_vector<T, 2><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
           case 4: k_spmv_csr_vector<T, 4><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
           case 8: k_spmv_csr_vector<T, 8><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;

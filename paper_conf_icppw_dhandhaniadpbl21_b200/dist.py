@@ -1,0 +1,173 @@
+"""Multi-GPU drivers (one process per GPU, torch.distributed over NCCL; gloo for the CPU tests).
+
+The labelling pass shards in the two ways SURVEY §8(e) names:
+
+1. Corpus sharding (independent units, "scaling: weak" in bench.py; strong-scaling helper here):
+   matrices are assigned to ranks by LPT on an estimated cost, each rank labels its shard with
+   ``sfs_label_corpus`` and the fixed-size result rows are gathered once (``all_gather_into_tensor``).
+   The paper labels one platform at a time (§5.1); sharding the M×F×N experiments of P:L46
+   over GPUs is the build's addition.
+2. Row partition of one large matrix (one exchange per SpMV): rank k holds the contiguous row block
+   A[r_k:r_{k+1}, :] with global column ids; each SpMV is ``all_gather_into_tensor(x_full, x_local)``
+   followed by the local ``sfs_spmv``.
+
+Everything that touches matrix data runs in libsfs; this module only partitions, launches and
+gathers.  The labeller / SpMV callables are injectable so the host logic is testable with gloo on CPU.
+"""
+from __future__ import annotations
+
+import heapq
+from dataclasses import dataclass
+from typing import Callable, Dict, List, Optional, Sequence
+
+import numpy as np
+
+# ------------------------------------------------------------------ corpus sharding
+
+
+def lpt_assign(costs: Sequence[float], world: int) -> List[List[int]]:
+    """Longest-processing-time-first: items in decreasing cost (ties by index) each go to the least
+    loaded rank (ties to the lowest rank).  Deterministic, identical on every rank; each shard is
+    returned in increasing item order."""
+    heap = [(0.0, r) for r in range(world)]
+    shards: List[List[int]] = [[] for _ in range(world)]
+    for i in sorted(range(len(costs)), key=lambda j: (-costs[j], j)):
+        load, r = heapq.heappop(heap)
+        shards[r].append(i)
+        heapq.heappush(heap, (load + float(costs[i]), r))
+    return [sorted(s) for s in shards]
+
+
+# fixed-size result row gathered across ranks: id, label, matrix status, admissible mask, csr variant,
+# t_spmv[5], t_convert[5], status[5], t_features, 23 features  -> 44 float64
+RESULT_FIELDS = 44
+
+
+def pack_result(i: int, feat: dict, lab: dict) -> np.ndarray:
+    from . import FEATURE_FLOAT_FIELDS, FEATURE_INT_FIELDS
+    row = [i, lab["label"], lab["matrix_status"], lab["admissible_mask"], lab["csr_variant"]]
+    row += list(lab["t_spmv_us"]) + list(lab["t_convert_us"]) + list(lab["status"]) + [lab["t_features_us"]]
+    row += [feat[k] for k in FEATURE_INT_FIELDS] + [feat[k] for k in FEATURE_FLOAT_FIELDS]
+    assert len(row) == RESULT_FIELDS
+    return np.array(row, dtype=np.float64)
+
+
+def unpack_result(row: np.ndarray) -> dict:
+    from . import FEATURE_FLOAT_FIELDS, FEATURE_INT_FIELDS
+    r = row.tolist()
+    out = {"id": int(r[0]), "label": int(r[1]), "matrix_status": int(r[2]), "admissible_mask": int(r[3]),
+           "csr_variant": int(r[4]), "t_spmv_us": r[5:10], "t_convert_us": r[10:15],
+           "status": [int(v) for v in r[15:20]], "t_features_us": r[20]}
+    feats = {}
+    for j, k in enumerate(FEATURE_INT_FIELDS):
+        feats[k] = int(r[21 + j])
+    for j, k in enumerate(FEATURE_FLOAT_FIELDS):
+        feats[k] = r[21 + len(FEATURE_INT_FIELDS) + j]
+    out["features"] = feats
+    return out
+
+
+def gather_results(local_rows: np.ndarray, world: int, max_per_rank: int, device=None, group=None) -> np.ndarray:
+    """all_gather_into_tensor of fixed-size result rows, padded to max_per_rank (pad id = -1).
+    Returns every rank's valid rows, sorted by matrix id."""
+    import torch
+    import torch.distributed as dist
+    pad = np.full((max_per_rank, RESULT_FIELDS), -1.0)
+    pad[:len(local_rows)] = local_rows
+    t = torch.from_numpy(pad.reshape(-1)).to(device or "cpu")
+    if world == 1:
+        allr = t
+    else:
+        allr = torch.empty(world * t.numel(), dtype=t.dtype, device=t.device)
+        dist.all_gather_into_tensor(allr, t, group=group)
+    rows = allr.cpu().numpy().reshape(world * max_per_rank, RESULT_FIELDS)
+    rows = rows[rows[:, 0] >= 0]
+    return rows[np.argsort(rows[:, 0], kind="stable")]
+
+
+def label_corpus_sharded(ids: Sequence[int], costs: Sequence[float], make: Callable[[int], object],
+                         labeller: Callable[[list], tuple], rank: int, world: int, batch_bytes: float = 40e9,
+                         nbytes: Optional[Callable[[object], float]] = None, device=None, group=None) -> List[dict]:
+    """Strong-scaling corpus labelling: LPT-shard `ids` (costs aligned), build each matrix with
+    `make(id)`, label in memory-bounded batches with `labeller(list_of_matrices) -> (feats, labels)`
+    (``sfs.label_corpus`` on a GPU), then gather every rank's results.  Returns the results of ALL
+    matrices, in id order, on every rank."""
+    shards = lpt_assign(costs, world)
+    mine = [ids[j] for j in shards[rank]]
+    rows = []
+    batch, batch_ids, used = [], [], 0.0
+    for i in mine + [None]:
+        if i is not None:
+            A = make(i)
+            b = nbytes(A) if nbytes else 0.0
+        if batch and (i is None or used + b > batch_bytes):
+            feats, labs = labeller(batch)
+            rows += [pack_result(bi, f, L) for bi, f, L in zip(batch_ids, feats, labs)]
+            batch, batch_ids, used = [], [], 0.0
+        if i is not None:
+            batch.append(A)
+            batch_ids.append(i)
+            used += b
+    local = np.stack(rows) if rows else np.zeros((0, RESULT_FIELDS))
+    maxn = max(len(s) for s in shards)
+    return [unpack_result(r) for r in gather_results(local, world, maxn, device, group)]
+
+
+# ------------------------------------------------------------------ row partition of one matrix
+
+
+def row_blocks(m: int, world: int) -> List[int]:
+    """Equal contiguous row blocks of ceil(m / world) rows (the last may be short or empty)."""
+    b = -(-m // world)
+    return [min(m, k * b) for k in range(world + 1)]
+
+
+def slice_rows(rp: np.ndarray, col: np.ndarray, val: np.ndarray, r0: int, r1: int):
+    """Host CSR of rows [r0, r1) with global column ids."""
+    a, b = int(rp[r0]), int(rp[r1])
+    return (rp[r0:r1 + 1] - a).astype(np.int32), col[a:b].copy(), val[a:b].copy()
+
+
+@dataclass
+class RowPartition:
+    m: int
+    n: int
+    world: int
+    rank: int
+
+    @property
+    def bounds(self):
+        return row_blocks(self.m, self.world)
+
+    @property
+    def block(self) -> int:
+        return -(-self.m // self.world)
+
+    @property
+    def local_rows(self) -> int:
+        b = self.bounds
+        return b[self.rank + 1] - b[self.rank]
+
+
+def rowpart_spmv_iterate(part: RowPartition, local_spmv: Callable, x_local, iters: int, group=None,
+                         swap: bool = True):
+    """`iters` times: x_full = all_gather(x_local) (padded blocks), y_local = A_k x_full[:n]; if swap,
+    y_local becomes the next x_local (power-iteration pattern, square A).  Returns y_local.
+    `local_spmv(x_full_view, y_local)` runs the rank's SpMV (sfs_spmv on a GPU)."""
+    import torch
+    import torch.distributed as dist
+    blk = part.block
+    x_pad = torch.zeros(blk, dtype=x_local.dtype, device=x_local.device)
+    x_full = torch.empty(blk * part.world, dtype=x_local.dtype, device=x_local.device)
+    y_local = torch.empty(part.local_rows, dtype=x_local.dtype, device=x_local.device)
+    cur = x_local
+    for _ in range(iters):
+        x_pad[:cur.numel()].copy_(cur)
+        if part.world > 1:
+            dist.all_gather_into_tensor(x_full, x_pad, group=group)
+        else:
+            x_full.copy_(x_pad)
+        local_spmv(x_full[:part.n], y_local)
+        if swap:
+            cur = y_local.clone()
+    return y_local

@@ -1,0 +1,132 @@
+"""N > 1 host logic on CPU: world_size-2 gloo process groups (no GPU).  The labeller / local SpMV are
+test doubles backed by the oracle; on a GPU box they are sfs.label_corpus / sfs.spmv."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
+
+
+def test_lpt_assign():
+    costs = [5, 1, 9, 3, 3, 7, 2]
+    sh = sd.lpt_assign(costs, 3)
+    assert sorted(sum(sh, [])) == list(range(7))
+    loads = [sum(costs[i] for i in s) for s in sh]
+    assert max(loads) - min(loads) <= max(costs)
+    assert sd.lpt_assign(costs, 3) == sh  # deterministic
+    assert sd.lpt_assign([1.0] * 4, 1) == [[0, 1, 2, 3]]
+    assert sd.lpt_assign([], 2) == [[], []]
+
+
+def test_row_blocks():
+    assert sd.row_blocks(10, 4) == [0, 3, 6, 9, 10]
+    assert sd.row_blocks(8, 8) == list(range(9))
+    assert sd.row_blocks(3, 4) == [0, 1, 2, 3, 3]
+
+
+def test_pack_roundtrip():
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    feat = {k: i for i, k in enumerate(sfs.FEATURE_INT_FIELDS)}
+    feat.update({k: 0.5 + i for i, k in enumerate(sfs.FEATURE_FLOAT_FIELDS)})
+    lab = {"label": 3, "matrix_status": 0, "admissible_mask": 31, "csr_variant": 1, "t_spmv_us": [1, 2, 3, 4, 5],
+           "t_convert_us": [0, 1, 1, 1, 1], "status": [0, 0, -3, 0, -7], "t_features_us": 9.0}
+    r = sd.unpack_result(sd.pack_result(42, feat, lab))
+    assert r["id"] == 42 and r["label"] == 3 and r["status"] == [0, 0, -3, 0, -7]
+    assert all(r["features"][k] == feat[k] for k in feat)
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _oracle_labeller(batch):
+    import oracle
+    feats, labs = [], []
+    for (A, x) in batch:
+        lab, f, ts, tc = oracle.label_matrix(A.m, A.n, A.rp, A.col, A.val.astype(np.float64), x, reps=1)
+        f = dict(f)
+        f["csr_variant"] = 0
+        feats.append(f)
+        labs.append({"label": lab, "matrix_status": 0, "admissible_mask": f["admissible_mask"], "csr_variant": 0,
+                     "t_spmv_us": list(ts * 1e6), "t_convert_us": list(tc * 1e6),
+                     "status": [0 if (f["admissible_mask"] >> k) & 1 else -3 for k in range(5)],
+                     "t_features_us": 0.0})
+    return feats, labs
+
+
+def _make(i):
+    import sfsgen
+    s = sfsgen.make_spec(sfsgen.UNIFORM if i % 2 else sfsgen.BAND, seed=i + 1, m=300 + 37 * i, ia=3, pa=5.0)
+    A = sfsgen.generate(s)
+    return (A, sfsgen.vector(i, A.n))
+
+
+def _worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        ids = list(range(9))
+        costs = [float(_make(i)[0].nnz) for i in ids]
+        res = sd.label_corpus_sharded(ids, costs, _make, _oracle_labeller, rank, world, batch_bytes=2e4,
+                                      nbytes=lambda t: t[0].nbytes())
+        # row partition of one square matrix, 3 power-iteration steps
+        import oracle
+        import sfsgen
+        A = sfsgen.generate(sfsgen.make_spec(sfsgen.ST2D5, ia=13))
+        part = sd.RowPartition(A.m, A.n, world, rank)
+        b = part.bounds
+        rp, col, val = sd.slice_rows(A.rp, A.col, A.val, b[rank], b[rank + 1])
+
+        def local_spmv(xf, y):
+            yy, _ = oracle.spmv_csr(len(rp) - 1, A.n, rp, col, val, xf.numpy())
+            y.copy_(torch.from_numpy(yy))
+
+        x = torch.from_numpy(sfsgen.vector(5, A.n))
+        y = sd.rowpart_spmv_iterate(part, local_spmv, x[b[rank]:b[rank + 1]].clone(), iters=3)
+        q.put((rank, [(r["id"], r["label"], r["features"]["nnz"]) for r in res], y.numpy()))
+    except Exception as e:  # surface worker failures immediately
+        import traceback
+        q.put((rank, "ERROR", traceback.format_exc()))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_corpus_and_rowpartition():
+    import oracle
+    import sfsgen
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = [q.get(timeout=240) for _ in range(world)]
+    for o in out:
+        assert o[1] != "ERROR", o[2]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    out.sort()
+    (r0, res0, y0), (r1, res1, y1) = out
+    assert res0 == res1  # every rank holds the whole corpus result
+    assert [i for i, _, _ in res0] == list(range(9))
+    for i, lab, nnz in res0:
+        assert nnz == _make(i)[0].nnz and 0 <= lab < 5
+    # row-partitioned power iteration == global oracle SpMV iterated
+    A = sfsgen.generate(sfsgen.make_spec(sfsgen.ST2D5, ia=13))
+    x = sfsgen.vector(5, A.n)
+    for _ in range(3):
+        x, _ = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
+    y = np.concatenate([y0, y1])
+    assert np.allclose(y, x, rtol=1e-12, atol=0)
