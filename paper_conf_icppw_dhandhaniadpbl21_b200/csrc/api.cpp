@@ -354,6 +354,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       if (A->variant == 1) {
         A->work = own(csr_merge_work_bytes(m, z, d.dtype));
         if (!A->work) return bail(SFS_ERR_OOM, "csr merge carries");
+        TRY_CUDA(launch_csr_merge_prepare((const int*)A->ptr[0], m, z, A->work, s));
       }
       break;
     }
@@ -702,7 +703,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
       const int kpc = spmv_kernels_per_call(A);
       if (o.cold) {
         for (int r = 0; r < o.reps; r++) {
-          if (flush) { cudaMemsetAsync(flush, r & 0xff, flush_bytes, s); count_launch(); }
+          if (flush) launch_l2_flush(flush, flush_bytes, s);
           cudaEvent_t a = ev.get(), b = ev.get();
           cudaEventRecord(a, s);
           launch_spmv(A, x, y, s);

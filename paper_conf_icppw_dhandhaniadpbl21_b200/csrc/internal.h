@@ -96,8 +96,10 @@ struct Matrix;
 int spmv_kernels_per_call(const Matrix* A);
 cudaError_t launch_spmv(const Matrix* A, const void* x, void* y, cudaStream_t s);
 size_t csr_merge_work_bytes(long long m, long long z, int dtype);
+cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s);
 int csr_vector_tpv(long long m, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
+cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s);
 
 // ---------------------------------------------------------------- matrix handle
 struct Matrix {
