@@ -48,6 +48,7 @@ def parse():
     p.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--out", default=None, help="also append the JSON line to this file")
+    p.add_argument("--dump", default=None, help="write per-matrix results of the last timed step (JSONL)")
     return p.parse_args()
 
 
@@ -286,11 +287,19 @@ def run_ours(args):
     barrier()
     t_e2e = maxr(e2.elapsed_time(e3) / 1000.0)
     h2d = sum(m.nbytes() + m.x.numel() * m.x.element_size() for m in hmats)
-    e2e = {"value": world * n * args.e2e_steps / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d,
-           "d2h_bytes_per_step": n * DAGGR_BYTES}
+    e2e = None
+    if args.e2e_steps > 0:
+        e2e = {"value": world * n * args.e2e_steps / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d,
+               "d2h_bytes_per_step": n * DAGGR_BYTES}
 
     # ---- roofline of the dominant kernel (from the race's own CUDA events, inside the timed region)
     feats, labs = results[-1]
+    if args.dump and rank == 0:
+        import sfsgen
+        with open(args.dump, "w") as fh:
+            for (i, A, _), f, L in zip(host, feats, labs):
+                fh.write(json.dumps({"id": i, "spec": sfsgen.corpus_spec(200, i).describe(), "m": A.m, "nnz": A.nnz,
+                                     "features": f, "race": L}) + "\n")
     per_fmt = {}
     for f in range(sfs.NFMT):
         tt = sum(L["t_spmv_us"][f] for L in labs if L["status"][f] == 0) * args.reps

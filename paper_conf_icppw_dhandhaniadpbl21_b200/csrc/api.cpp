@@ -175,10 +175,10 @@ static void finalize(long long m, long long n, long long z, const DevAggr& a, lo
   if (f->ell_size <= lim) mask |= 1u << SFS_ELL;
   if (f->dia_size <= lim) mask |= 1u << SFS_DIA;
   f->admissible_mask = mask;
-  // Q17: CSR vector kernel unless row lengths are skewed
+  // Q17: CSR stream kernel (warp per 32 rows) unless row lengths are skewed, then merge path
   const long long avg = std::max(1LL, z / m);
-  f->csr_variant = (mx <= 4 * avg + 32) ? 0 : 1;
-  if (o.csr_variant == 0 || o.csr_variant == 1) f->csr_variant = o.csr_variant;
+  f->csr_variant = (mx <= 4 * avg + 32) ? 2 : 1;
+  if (o.csr_variant >= 0 && o.csr_variant <= 2) f->csr_variant = o.csr_variant;
 }
 
 static sfs_status check_csr(const sfs_csr* A) {

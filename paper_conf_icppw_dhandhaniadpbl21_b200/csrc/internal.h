@@ -109,7 +109,7 @@ struct Matrix {
   void* owned[8] = {nullptr};  // buffers to free
   int n_owned = 0;
   long long bytes = 0;
-  int variant = 0;             // CSR: 0 vector, 1 merge
+  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream
   void* work = nullptr;        // CSR merge carries
   cudaStream_t stream = nullptr;
 };

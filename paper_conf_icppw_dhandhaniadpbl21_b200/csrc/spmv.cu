@@ -5,16 +5,30 @@
 // cores: the path is not a dense contraction.  Products and sums are formed in fp64 for both value
 // types (an fp32 product is exact in fp64), so fp32 rows of ~10^5 entries stay within the 1e-5
 // per-row tolerance; y is rounded once to its dtype.
+//
+// Two regimes shape every launch: matrices far larger than the GPU's in-flight capacity are
+// bandwidth-bound (one wave, each thread streaming a long slice); L2-resident / mid-size matrices
+// are latency-bound, so the work of a row group is split S ways (ELL slots, DIA diagonals, CSR
+// windows) and the partial sums are combined in shared memory, keeping each thread to one or two
+// dependent memory round trips.  Back-to-back SpMVs (the race's 100 reps) use programmatic
+// dependent launch: each kernel waits (griddepcontrol.wait) before touching memory, and releases
+// its successor (griddepcontrol.launch_dependents) when its work is issued, hiding launch latency
+// without overlapping two SpMVs' memory traffic.
 //   CSR vector : TPV lanes per row (TPV from floor(z/m)), grid of 148*64 warps (the csr_max
-//                feature, Q4), shuffle reduction.
+//                feature, Q4), shuffle reduction.  Kept as the CUSP-mapping variant.
+//   CSR stream : warp-groups of 32 consecutive rows; windows of their contiguous nnz streamed with
+//                coalesced loads, products staged in smem, lane j sums row j.  S warps per group.
 //   CSR merge  : merge-path tiles over (row ends + nnz), products staged in smem, block-wide
 //                segmented scan of thread carries, one carry per tile added by a fix-up kernel.
-//   COO        : each warp owns a contiguous range of 128-item chunks (4 items per lane, 128-bit
+//   COO        : each warp owns a contiguous range of 256-item chunks (8 items per lane, 128-bit
 //                loads), warp segmented reduction by row; rows are stored directly except the
 //                range's first row and its final carry (atomicAdd).
-//   ELL / HYB  : 4 rows per thread, column-major slab read with 128-bit loads (coalesced per slot);
-//                HYB = ELL part (writes y) then COO part (accumulates).
-//   DIA        : 4 rows per thread, slab read with 128-bit loads, x through L1.
+//   ELL / HYB  : 4 rows per thread, column-major slab read with 128-bit loads (coalesced per slot),
+//                S slot-parts per row group; HYB = ELL part (writes y) then COO part (accumulates).
+//   DIA        : 4 (fp64) / 8 (fp32) rows per thread 256 apart (coalesced slab and x), S diagonal
+//                parts per row block.
+#include <stdlib.h>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -22,6 +36,65 @@ namespace sfs {
 namespace {
 
 typedef double acc_t;
+
+constexpr long long kResidentThreads = (long long)kSMs * 2048;
+
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+
+bool pdl_enabled() {
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SFS_PDL");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
+
+// cudaLaunchKernelEx with the programmatic-stream-serialization attribute (PDL).
+template <typename... Params, typename... Args>
+cudaError_t launch_k(void (*kern)(Params...), dim3 grid, dim3 block, cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  count_launch();
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<Params>(args)...);
+}
+
+int grid_cap(long long items, int threads, int per_sm) {
+  long long g = ceil_div(items, threads), cap = (long long)kSMs * per_sm;
+  return (int)(g > cap ? cap : (g < 1 ? 1 : g));
+}
+
+int pow2_ceil(long long v) {
+  int p = 1;
+  while (p < v && p < (1 << 20)) p <<= 1;
+  return p;
+}
+
+// Split factor for a latency-bound launch: enough parts that each thread does <= `per_thread` units
+// of `units` (slots, diagonals, windows), but stop once `items * S` threads would exceed `fill` x the
+// GPU's resident threads (bandwidth-bound sizes keep S = 1).
+int split_factor(long long items, long long units, long long per_thread, int smax, long long fill = 2) {
+  int S = 1;
+  while (S < smax && ceil_div(units, S) > per_thread && items * S * 2 <= fill * kResidentThreads) S <<= 1;
+  return S;
+}
+
+template <typename T>
+__global__ void k_zero(T* __restrict__ y, long long m) {
+  pdl_wait();
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (long long)gridDim.x * blockDim.x)
+    y[i] = T(0);
+  pdl_trigger();
+}
 
 // ======================================================================== CSR vector
 // Vector v (TPV lanes) owns rows v, v+V, v+2V, ... (V = vectors in the grid): the CUSP-style mapping
@@ -46,6 +119,7 @@ template <typename T, int TPV>
 __global__ void __launch_bounds__(256) k_spmv_csr_vector(const int* __restrict__ rp, const int* __restrict__ col,
                                                          const T* __restrict__ val, const T* __restrict__ x,
                                                          T* __restrict__ y, long long m) {
+  pdl_wait();
   const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const int lane = threadIdx.x & (TPV - 1);
   const long long V = ((long long)gridDim.x * blockDim.x) / TPV;
@@ -72,6 +146,86 @@ __global__ void __launch_bounds__(256) k_spmv_csr_vector(const int* __restrict__
     }
     b0 = nb0; e0 = ne0; b1 = nb1; e1 = ne1;
   }
+  pdl_trigger();
+}
+
+// ======================================================================== CSR stream (regular rows)
+// A group of 32 consecutive rows has contiguous nnz [rp[r0], rp[r0+32]).  S warps share a group:
+// warp part p streams windows p, p+S, ... of kSW items (lane i loads items i, i+32, ...: every load
+// instruction is one contiguous 128/256 B request), stages the products in its own smem window, and
+// lane j adds row r0+j's part of the window.  The S partial sums meet in shared memory.
+constexpr int kSThreads = 256;
+constexpr int kSWarps = kSThreads / 32;
+template <typename T> constexpr int stream_u() { return sizeof(T) == 4 ? 16 : 8; }  // items per lane per window
+template <typename T> constexpr int stream_ctas() { return sizeof(T) == 4 ? 3 : 4; }  // register cap
+constexpr int kSWMax = 32 * 16;
+
+template <typename T>
+__global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream(const int* __restrict__ rp,
+                                                               const int* __restrict__ col,
+                                                               const T* __restrict__ val, const T* __restrict__ x,
+                                                               T* __restrict__ y, long long m, int S) {
+  constexpr int kSU = stream_u<T>();  // all of a lane's loads of a window are in flight together
+  constexpr int kSW = 32 * kSU;
+  __shared__ acc_t sbuf[kSWarps][kSWMax];
+  __shared__ acc_t s_part[kSWarps][32];
+  pdl_wait();
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  const int NG = kSWarps / S;  // groups per CTA iteration
+  const int p = w / NG, gl = w % NG;
+  acc_t* buf = sbuf[w];
+  const long long ngroups = ceil_div(m, 32);
+  const long long niter = ceil_div(ngroups, NG);
+  for (long long it = blockIdx.x; it < niter; it += gridDim.x) {
+    const long long g = it * NG + gl;
+    const long long r = g * 32 + lane;
+    const int b = g < ngroups ? __ldg(rp + (r < m ? r : m)) : 0;
+    const int e = g < ngroups ? __ldg(rp + (r < m ? r + 1 : m)) : 0;
+    const int s0 = __shfl_sync(0xffffffffu, b, 0), s1 = __shfl_sync(0xffffffffu, e, 31);
+    acc_t acc = 0;
+    for (int w0 = s0 + p * kSW; w0 < s1; w0 += S * kSW) {
+      const int n = s1 - w0 < kSW ? s1 - w0 : kSW;
+      int c[kSU];
+      T v[kSU];
+#pragma unroll
+      for (int u = 0; u < kSU; u++) {
+        const int i = u * 32 + lane;
+        if (i < n) {
+          c[u] = ld_stream(col + w0 + i);
+          v[u] = ld_stream(val + w0 + i);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < kSU; u++) {
+        const int i = u * 32 + lane;
+        if (i < n) buf[i] = (acc_t)v[u] * (acc_t)ld_x(x + c[u]);
+      }
+      __syncwarp();
+      const int lo = (b > w0 ? b : w0) - w0, hi = (e < w0 + n ? e : w0 + n) - w0;
+      acc_t a0 = 0, a1 = 0;
+      int i = lo;
+      for (; i + 1 < hi; i += 2) {
+        a0 += buf[i];
+        a1 += buf[i + 1];
+      }
+      if (i < hi) a0 += buf[i];
+      acc += a0 + a1;
+      __syncwarp();
+    }
+    if (S == 1) {
+      if (g < ngroups && r < m) y[r] = (T)acc;
+    } else {
+      s_part[w][lane] = acc;
+      __syncthreads();
+      if (p == 0) {
+        acc_t t = acc;
+        for (int q = 1; q < S; q++) t += s_part[q * NG + gl][lane];
+        if (g < ngroups && r < m) y[r] = (T)t;
+      }
+      __syncthreads();
+    }
+  }
+  pdl_trigger();
 }
 
 // ======================================================================== CSR merge path
@@ -147,14 +301,43 @@ __global__ void __launch_bounds__(kMT) k_spmv_csr_merge(const int* __restrict__ 
   __shared__ acc_t s_prod[kMTile];
   __shared__ acc_t s_ws[33];
   __shared__ int s_wf[32];
+  pdl_wait();
   const long long total = m + z;
   const long long d0 = (long long)blockIdx.x * kMTile;
   const long long d1 = d0 + kMTile < total ? d0 + kMTile : total;
   const int2 c0 = __ldg(coords + blockIdx.x), c1 = __ldg(coords + blockIdx.x + 1);
   const int r0 = c0.x, k0 = c0.y, r1 = c1.x, k1 = c1.y;
-  for (int i = threadIdx.x; i <= r1 - r0 + 1 && r0 + i <= m; i += kMT) s_rp[i] = __ldg(rp + r0 + i);
-  for (int i = threadIdx.x; i < k1 - k0; i += kMT)
-    s_prod[i] = (acc_t)ld_stream(val + k0 + i) * (acc_t)ld_x(x + ld_stream(col + k0 + i));
+  // Load phase, fully unrolled so every thread has all of its loads in flight at once: row ends of
+  // the tile, then col/val of its nnz (coalesced: item u*kMT + tid), then the x gathers.
+  {
+    const int nr = (r1 - r0 + 2 < (int)(m - r0 + 1)) ? r1 - r0 + 2 : (int)(m - r0 + 1);
+    const int nk = k1 - k0;
+    int rv[kMI + 1], cv[kMI];
+    T vv[kMI];
+#pragma unroll
+    for (int u = 0; u <= kMI; u++) {
+      const int i = threadIdx.x + u * kMT;
+      if (i < nr) rv[u] = __ldg(rp + r0 + i);
+    }
+#pragma unroll
+    for (int u = 0; u < kMI; u++) {
+      const int i = threadIdx.x + u * kMT;
+      if (i < nk) {
+        cv[u] = ld_stream(col + k0 + i);
+        vv[u] = ld_stream(val + k0 + i);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u <= kMI; u++) {
+      const int i = threadIdx.x + u * kMT;
+      if (i < nr) s_rp[i] = rv[u];
+    }
+#pragma unroll
+    for (int u = 0; u < kMI; u++) {
+      const int i = threadIdx.x + u * kMT;
+      if (i < nk) s_prod[i] = (acc_t)vv[u] * (acc_t)ld_x(x + cv[u]);
+    }
+  }
   __syncthreads();
   const int ld = threadIdx.x * kMI;
   const int items_all = (int)(d1 - d0);
@@ -187,16 +370,19 @@ __global__ void __launch_bounds__(kMT) k_spmv_csr_merge(const int* __restrict__ 
     carry_row[blockIdx.x] = r1;  // row open at the tile end (r1 == m: none)
     carry_val[blockIdx.x] = tile_total;
   }
+  pdl_trigger();
 }
 
 template <typename T>
 __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const acc_t* __restrict__ carry_val,
                                        long long tiles, long long m, T* __restrict__ y) {
+  pdl_wait();
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < tiles; t += (long long)gridDim.x * blockDim.x) {
     const int r = carry_row[t];
     const acc_t v = carry_val[t];
     if (r < m && v != 0) atomicAdd(y + r, (T)v);
   }
+  pdl_trigger();
 }
 
 // ======================================================================== COO (also the COO part of HYB)
@@ -215,201 +401,254 @@ template <typename T, bool ACCUM>
 __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
                                                           T* __restrict__ y, long long z, long long chunks_per_warp) {
+  pdl_wait();
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kChunk);
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long cb = warp * chunks_per_warp;
   const long long ce = cb + chunks_per_warp < nchunks ? cb + chunks_per_warp : nchunks;
-  if (cb >= ce) return;
-  const int last_row = __ldg(row + z - 1);
-  const int range_first = __ldg(row + cb * kChunk);
-  int carry_row = -1;
-  acc_t carry = 0;
-  for (long long ch = cb; ch < ce; ch++) {
-    const long long k = ch * kChunk + l * kCooV;
-    int r[kCooV];
-    acc_t p[kCooV];
-    if (k + kCooV <= z) {
-      int c[kCooV];
-      T v[kCooV];
+  if (cb < ce) {
+    const int last_row = __ldg(row + z - 1);
+    const int range_first = __ldg(row + cb * kChunk);
+    int carry_row = -1;
+    acc_t carry = 0;
+    for (long long ch = cb; ch < ce; ch++) {
+      const long long k = ch * kChunk + l * kCooV;
+      int r[kCooV];
+      acc_t p[kCooV];
+      if (k + kCooV <= z) {
+        int c[kCooV];
+        T v[kCooV];
 #pragma unroll
-      for (int q = 0; q < kCooV / 4; q++) {
-        const int4 rr = ld_stream4(row + k + 4 * q), cc = ld_stream4(col + k + 4 * q);
-        Vec4<T> vv;
-        vv.load_stream(val + k + 4 * q);
-        r[4 * q] = rr.x; r[4 * q + 1] = rr.y; r[4 * q + 2] = rr.z; r[4 * q + 3] = rr.w;
-        c[4 * q] = cc.x; c[4 * q + 1] = cc.y; c[4 * q + 2] = cc.z; c[4 * q + 3] = cc.w;
+        for (int q = 0; q < kCooV / 4; q++) {
+          const int4 rr = ld_stream4(row + k + 4 * q), cc = ld_stream4(col + k + 4 * q);
+          Vec4<T> vv;
+          vv.load_stream(val + k + 4 * q);
+          r[4 * q] = rr.x; r[4 * q + 1] = rr.y; r[4 * q + 2] = rr.z; r[4 * q + 3] = rr.w;
+          c[4 * q] = cc.x; c[4 * q + 1] = cc.y; c[4 * q + 2] = cc.z; c[4 * q + 3] = cc.w;
 #pragma unroll
-        for (int i = 0; i < 4; i++) v[4 * q + i] = vv.v[i];
-      }
+          for (int i = 0; i < 4; i++) v[4 * q + i] = vv.v[i];
+        }
 #pragma unroll
-      for (int i = 0; i < kCooV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
-    } else {
+        for (int i = 0; i < kCooV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
+      } else {
 #pragma unroll
-      for (int i = 0; i < kCooV; i++) {
-        if (k + i < z) {
-          r[i] = ld_stream(row + k + i);
-          p[i] = (acc_t)ld_stream(val + k + i) * (acc_t)ld_x(x + ld_stream(col + k + i));
-        } else {
-          r[i] = last_row;  // padding joins the last segment with value 0
-          p[i] = 0;
+        for (int i = 0; i < kCooV; i++) {
+          if (k + i < z) {
+            r[i] = ld_stream(row + k + i);
+            p[i] = (acc_t)ld_stream(val + k + i) * (acc_t)ld_x(x + ld_stream(col + k + i));
+          } else {
+            r[i] = last_row;  // padding joins the last segment with value 0
+            p[i] = 0;
+          }
         }
       }
-    }
-    const int rf = r[0], rl = r[kCooV - 1];
-    // the previous chunk's carry ends exactly at this chunk boundary: emit it
-    const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
-    if (carry_row >= 0 && carry_row != chunk_first) {
-      if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, carry_row == range_first);
-      carry_row = -1;
-      carry = 0;
-    }
-    // lane-local segments: head (row rf), middles (complete), tail (row rl)
-    acc_t head = p[0], cur = p[0];
-    int cr = rf;
-    bool in_head = true;
-#pragma unroll
-    for (int i = 1; i < kCooV; i++) {
-      if (r[i] != cr) {
-        if (in_head) { head = cur; in_head = false; }
-        else coo_emit<T, ACCUM>(y, cr, cur, cr == range_first);
-        cr = r[i];
-        cur = p[i];
-      } else {
-        cur += p[i];
+      const int rf = r[0], rl = r[kCooV - 1];
+      // the previous chunk's carry ends exactly at this chunk boundary: emit it
+      const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
+      if (carry_row >= 0 && carry_row != chunk_first) {
+        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, carry_row == range_first);
+        carry_row = -1;
+        carry = 0;
       }
-    }
-    if (in_head) head = cur;
-    const bool single = (rf == rl);
-    const acc_t in0 = (carry_row == rf) ? carry : acc_t(0);  // carry into lane 0 (same row)
-    // segmented scan of tails across lanes: S_l = f_l ? tail_l : S_{l-1} + tail_l
-    const int prev_rl = __shfl_up_sync(0xffffffffu, rl, 1);
-    int f = (l == 0) || !single || (prev_rl != rf);
-    acc_t S = cur + ((l == 0 && single) ? in0 : acc_t(0));
+      // lane-local segments: head (row rf), middles (complete), tail (row rl)
+      acc_t head = p[0], cur = p[0];
+      int cr = rf;
+      bool in_head = true;
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      acc_t us = __shfl_up_sync(0xffffffffu, S, o);
-      int uf = __shfl_up_sync(0xffffffffu, f, o);
-      if (l >= o) {
-        if (!f) S += us;
-        f |= uf;
+      for (int i = 1; i < kCooV; i++) {
+        if (r[i] != cr) {
+          if (in_head) { head = cur; in_head = false; }
+          else coo_emit<T, ACCUM>(y, cr, cur, cr == range_first);
+          cr = r[i];
+          cur = p[i];
+        } else {
+          cur += p[i];
+        }
       }
+      if (in_head) head = cur;
+      const bool single = (rf == rl);
+      const acc_t in0 = (carry_row == rf) ? carry : acc_t(0);  // carry into lane 0 (same row)
+      // segmented scan of tails across lanes: S_l = f_l ? tail_l : S_{l-1} + tail_l
+      const int prev_rl = __shfl_up_sync(0xffffffffu, rl, 1);
+      int f = (l == 0) || !single || (prev_rl != rf);
+      acc_t S = cur + ((l == 0 && single) ? in0 : acc_t(0));
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        acc_t us = __shfl_up_sync(0xffffffffu, S, o);
+        int uf = __shfl_up_sync(0xffffffffu, f, o);
+        if (l >= o) {
+          if (!f) S += us;
+          f |= uf;
+        }
+      }
+      const acc_t S_prev = __shfl_up_sync(0xffffffffu, S, 1);
+      const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
+      if (!single) {
+        const acc_t h = head + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0)));
+        coo_emit<T, ACCUM>(y, rf, h, rf == range_first);
+      }
+      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, rl == range_first);
+      carry_row = __shfl_sync(0xffffffffu, rl, 31);  // the chunk's last row stays open
+      carry = __shfl_sync(0xffffffffu, S, 31);
     }
-    const acc_t S_prev = __shfl_up_sync(0xffffffffu, S, 1);
-    const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
-    if (!single) {
-      const acc_t h = head + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0)));
-      coo_emit<T, ACCUM>(y, rf, h, rf == range_first);
-    }
-    if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, rl == range_first);
-    carry_row = __shfl_sync(0xffffffffu, rl, 31);  // the chunk's last row stays open
-    carry = __shfl_sync(0xffffffffu, S, 31);
+    if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
   }
-  if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
+  pdl_trigger();
 }
 
 // ======================================================================== ELL (and the ELL part of HYB)
-// Thread = 4 consecutive rows; slots are read in batches of 4 (four 16 B col vectors and four 16/32 B
-// val vectors issued before any x gather), grid of one wave striding over row groups.
+// Thread = 4 consecutive rows x one of S slot-parts; slots are read in batches (four / eight 16 B col
+// vectors and as many 16/32 B val vectors issued before any x gather).  CTA = S parts x G row
+// groups (a warp = 32 consecutive groups of one part); parts meet in shared memory.
 constexpr int kEllThreads = 256;
-constexpr int kEllBatch = 4;
+template <typename T> constexpr int ell_batch() { return sizeof(T) == 4 ? 8 : 4; }   // bytes in flight per thread
+template <typename T> constexpr int ell_ctas() { return sizeof(T) == 4 ? 3 : 4; }    // CTAs / SM (register cap)
 
 template <typename T>
-__global__ void __launch_bounds__(kEllThreads, 4) k_spmv_ell(const int* __restrict__ ecol, const T* __restrict__ eval,
-                                                             const T* __restrict__ x, T* __restrict__ y, long long m,
-                                                             long long P, int K) {
+__global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
+                                                                         const T* __restrict__ eval,
+                                                                         const T* __restrict__ x, T* __restrict__ y,
+                                                                         long long m, long long P, int K, int S) {
+  constexpr int kB = ell_batch<T>();
+  __shared__ acc_t s_part[kEllThreads][4];
+  pdl_wait();
+  const int G = kEllThreads / S;
+  const int p = threadIdx.x / G, g = threadIdx.x % G;
+  const int Kp = (K + S - 1) / S;
+  const int j0 = p * Kp, j1 = j0 + Kp < K ? j0 + Kp : K;
   const long long groups = P / 4;
-  for (long long g = (long long)blockIdx.x * blockDim.x + threadIdx.x; g < groups; g += (long long)gridDim.x * blockDim.x) {
-    const long long r = g * 4;
+  const long long niter = ceil_div(groups, G);
+  for (long long it = blockIdx.x; it < niter; it += gridDim.x) {
+    const long long grp = it * G + g;
+    const long long r = grp * 4;
     acc_t acc[4] = {0, 0, 0, 0};
-    const int* cp = ecol + r;
-    const T* vp = eval + r;
-    int j = 0;
-    for (; j + kEllBatch <= K; j += kEllBatch) {
-      int4 c[kEllBatch];
-      Vec4<T> v[kEllBatch];
+    if (grp < groups) {
+      const int* cp = ecol + r;
+      const T* vp = eval + r;
+      int j = j0;
+      for (; j + kB <= j1; j += kB) {
+        int4 c[kB];
+        Vec4<T> v[kB];
 #pragma unroll
-      for (int u = 0; u < kEllBatch; u++) {
-        c[u] = ld_stream4(cp + (long long)(j + u) * P);
-        v[u].load_stream(vp + (long long)(j + u) * P);
+        for (int u = 0; u < kB; u++) {
+          c[u] = ld_stream4(cp + (long long)(j + u) * P);
+          v[u].load_stream(vp + (long long)(j + u) * P);
+        }
+#pragma unroll
+        for (int u = 0; u < kB; u++) {
+          if (c[u].x >= 0) acc[0] += (acc_t)v[u].v[0] * (acc_t)ld_x(x + c[u].x);
+          if (c[u].y >= 0) acc[1] += (acc_t)v[u].v[1] * (acc_t)ld_x(x + c[u].y);
+          if (c[u].z >= 0) acc[2] += (acc_t)v[u].v[2] * (acc_t)ld_x(x + c[u].z);
+          if (c[u].w >= 0) acc[3] += (acc_t)v[u].v[3] * (acc_t)ld_x(x + c[u].w);
+        }
       }
-#pragma unroll
-      for (int u = 0; u < kEllBatch; u++) {
-        if (c[u].x >= 0) acc[0] += (acc_t)v[u].v[0] * (acc_t)ld_x(x + c[u].x);
-        if (c[u].y >= 0) acc[1] += (acc_t)v[u].v[1] * (acc_t)ld_x(x + c[u].y);
-        if (c[u].z >= 0) acc[2] += (acc_t)v[u].v[2] * (acc_t)ld_x(x + c[u].z);
-        if (c[u].w >= 0) acc[3] += (acc_t)v[u].v[3] * (acc_t)ld_x(x + c[u].w);
+      for (; j < j1; j++) {
+        const int4 c = ld_stream4(cp + (long long)j * P);
+        Vec4<T> v;
+        v.load_stream(vp + (long long)j * P);
+        if (c.x >= 0) acc[0] += (acc_t)v.v[0] * (acc_t)ld_x(x + c.x);
+        if (c.y >= 0) acc[1] += (acc_t)v.v[1] * (acc_t)ld_x(x + c.y);
+        if (c.z >= 0) acc[2] += (acc_t)v.v[2] * (acc_t)ld_x(x + c.z);
+        if (c.w >= 0) acc[3] += (acc_t)v.v[3] * (acc_t)ld_x(x + c.w);
       }
     }
-    for (; j < K; j++) {
-      const int4 c = ld_stream4(cp + (long long)j * P);
-      Vec4<T> v;
-      v.load_stream(vp + (long long)j * P);
-      if (c.x >= 0) acc[0] += (acc_t)v.v[0] * (acc_t)ld_x(x + c.x);
-      if (c.y >= 0) acc[1] += (acc_t)v.v[1] * (acc_t)ld_x(x + c.y);
-      if (c.z >= 0) acc[2] += (acc_t)v.v[2] * (acc_t)ld_x(x + c.z);
-      if (c.w >= 0) acc[3] += (acc_t)v.v[3] * (acc_t)ld_x(x + c.w);
-    }
+    if (S > 1) {
 #pragma unroll
-    for (int q = 0; q < 4; q++)
-      if (r + q < m) y[r + q] = (T)acc[q];
+      for (int q = 0; q < 4; q++) s_part[threadIdx.x][q] = acc[q];
+      __syncthreads();
+      if (p == 0) {
+        for (int pp = 1; pp < S; pp++)
+#pragma unroll
+          for (int q = 0; q < 4; q++) acc[q] += s_part[pp * G + g][q];
+      }
+      __syncthreads();
+    }
+    if (p == 0 && grp < groups) {
+#pragma unroll
+      for (int q = 0; q < 4; q++)
+        if (r + q < m) y[r + q] = (T)acc[q];
+    }
   }
+  pdl_trigger();
 }
 
 // ======================================================================== DIA
+// Thread t of a part owns rows R0 + t + Gq (q < 4 for fp64, 8 for fp32, G = 256/S threads per part):
+// for every diagonal a warp reads 32 consecutive slab entries and 32 consecutive x entries (coalesced
+// whatever the offset's alignment), 4 diagonals per batch, so each thread keeps 16 / 32 independent
+// loads in flight.  The S diagonal-parts of a row block meet in shared memory.
 constexpr int kDiaThreads = 256;
 constexpr int kDiaSmemOffs = 1024;
+template <typename T> constexpr int dia_rows() { return sizeof(T) == 4 ? 8 : 4; }
+template <typename T> constexpr int dia_ctas() { return sizeof(T) == 4 ? 2 : 3; }  // register cap
 constexpr int kDiaBatch = 4;
 
 template <typename T>
-__device__ __forceinline__ void dia_accum(acc_t* acc, const Vec4<T>& v, const T* __restrict__ x, long long c0,
-                                          long long n) {
-  if (c0 >= 0 && c0 + 3 < n) {
-    acc[0] += (acc_t)v.v[0] * (acc_t)ld_x(x + c0);
-    acc[1] += (acc_t)v.v[1] * (acc_t)ld_x(x + c0 + 1);
-    acc[2] += (acc_t)v.v[2] * (acc_t)ld_x(x + c0 + 2);
-    acc[3] += (acc_t)v.v[3] * (acc_t)ld_x(x + c0 + 3);
-  } else {
-#pragma unroll
-    for (int q = 0; q < 4; q++)
-      if (c0 + q >= 0 && c0 + q < n) acc[q] += (acc_t)v.v[q] * (acc_t)ld_x(x + c0 + q);
-  }
-}
-
-template <typename T>
-__global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia(const int* __restrict__ offs, const T* __restrict__ dval,
-                                                             const T* __restrict__ x, T* __restrict__ y, long long m,
-                                                             long long n, long long P, int nd) {
+__global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const int* __restrict__ offs,
+                                                                         const T* __restrict__ dval,
+                                                                         const T* __restrict__ x, T* __restrict__ y,
+                                                                         long long m, long long n, long long P, int nd,
+                                                                         int S) {
+  constexpr int kR = dia_rows<T>();
   __shared__ int s_off[kDiaSmemOffs];
+  __shared__ acc_t s_part[kDiaThreads * kR];
+  pdl_wait();
   const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
   for (int i = threadIdx.x; i < nsm; i += blockDim.x) s_off[i] = offs[i];
   __syncthreads();
-  const long long groups = P / 4;
-  for (long long g = (long long)blockIdx.x * blockDim.x + threadIdx.x; g < groups; g += (long long)gridDim.x * blockDim.x) {
-    const long long r = g * 4;
-    acc_t acc[4] = {0, 0, 0, 0};
-    const T* vp = dval + r;
-    int d = 0;
-    for (; d + kDiaBatch <= nd; d += kDiaBatch) {
-      Vec4<T> v[kDiaBatch];
+  const int G = kDiaThreads / S;
+  const int p = threadIdx.x / G, g = threadIdx.x % G;
+  const int Dp = (nd + S - 1) / S;
+  const int d0 = p * Dp, d1 = d0 + Dp < nd ? d0 + Dp : nd;
+  const long long rows_per_blk = (long long)G * kR;
+  const long long nblk = ceil_div(m, rows_per_blk);
+  for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+    const long long r0 = blk * rows_per_blk + g;
+    acc_t acc[kR];
 #pragma unroll
-      for (int u = 0; u < kDiaBatch; u++) v[u].load_stream(vp + (long long)(d + u) * P);
+    for (int q = 0; q < kR; q++) acc[q] = 0;
+    for (int d = d0; d < d1; d += kDiaBatch) {
+      T v[kDiaBatch][kR];
+      int off[kDiaBatch];
 #pragma unroll
       for (int u = 0; u < kDiaBatch; u++) {
-        const long long off = d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u);
-        dia_accum<T>(acc, v[u], x, r + off, n);
+        off[u] = d + u < d1 ? (d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u)) : 0;
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          const long long rr = r0 + (long long)q * G;
+          v[u][q] = (d + u < d1 && rr < m) ? ld_stream(dval + (long long)(d + u) * P + rr) : T(0);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < kDiaBatch; u++) {
+#pragma unroll
+        for (int q = 0; q < kR; q++) {
+          const long long c = r0 + (long long)q * G + (long long)off[u];
+          if (d + u < d1 && c >= 0 && c < n) acc[q] += (acc_t)v[u][q] * (acc_t)ld_x(x + c);
+        }
       }
     }
-    for (; d < nd; d++) {
-      Vec4<T> v;
-      v.load_stream(vp + (long long)d * P);
-      const long long off = d < kDiaSmemOffs ? s_off[d] : __ldg(offs + d);
-      dia_accum<T>(acc, v, x, r + off, n);
-    }
+    if (S > 1) {
 #pragma unroll
-    for (int q = 0; q < 4; q++)
-      if (r + q < m) y[r + q] = (T)acc[q];
+      for (int q = 0; q < kR; q++) s_part[threadIdx.x * kR + q] = acc[q];
+      __syncthreads();
+      if (p == 0) {
+        for (int pp = 1; pp < S; pp++)
+#pragma unroll
+          for (int q = 0; q < kR; q++) acc[q] += s_part[(pp * G + g) * kR + q];
+      }
+      __syncthreads();
+    }
+    if (p == 0) {
+#pragma unroll
+      for (int q = 0; q < kR; q++) {
+        const long long rr = r0 + (long long)q * G;
+        if (rr < m) y[rr] = (T)acc[q];
+      }
+    }
   }
+  pdl_trigger();
 }
 
 struct MergeWork {
@@ -429,90 +668,99 @@ MergeWork merge_work(void* base, long long tiles) {
   return w;
 }
 
-int grid_cap(long long items, int threads, int per_sm) {
-  long long g = ceil_div(items, threads), cap = (long long)kSMs * per_sm;
-  return (int)(g > cap ? cap : (g < 1 ? 1 : g));
-}
-
-// COO launch geometry: contiguous chunk ranges, at most 148*16 CTAs of 8 warps.
+// COO launch geometry: contiguous chunk ranges, one resident wave of warps at most.
 template <typename T, bool ACCUM>
-void launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
+cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
   const long long nchunks = ceil_div(z, kChunk);
-  const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);  // one resident wave (<= 64 regs)
+  const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);  // <= 64 regs: 4 CTAs / SM
   const long long cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
   const long long warps = ceil_div(nchunks, cpw);
   const unsigned blocks = (unsigned)ceil_div(warps, kCooThreads / 32);
-  k_spmv_coo<T, ACCUM><<<blocks, kCooThreads, 0, s>>>(row, col, val, x, y, z, cpw);
+  return launch_k(k_spmv_coo<T, ACCUM>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
+}
+
+template <typename T>
+cudaError_t launch_zero(T* y, long long m, cudaStream_t s) {
+  return launch_k(k_zero<T>, dim3(grid_cap(m, 256, 8)), dim3(256), s, y, m);
+}
+
+template <typename T>
+cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s) {
+  const long long groups = A->pitch / 4;
+  const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
+  const long long niter = ceil_div(groups, kEllThreads / S);
+  const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
+  return launch_k(k_spmv_ell<T>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1], x, y,
+                  A->m, A->pitch, K, S);
 }
 
 template <typename T>
 cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
   const long long m = A->m, z = A->nnz;
+  cudaError_t e = cudaSuccess;
   switch (A->fmt) {
     case SFS_CSR: {
       const int* rp = (const int*)A->ptr[0];
       const int* col = (const int*)A->ptr[1];
       const T* val = (const T*)A->ptr[2];
-      if (A->variant == 0) {
+      if (A->variant == 2) {
+        const long long groups = ceil_div(m, 32);
+        const long long windows = ceil_div(z, 32 * stream_u<T>());  // ~ windows over all groups
+        const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
+        const long long niter = ceil_div(groups, kSWarps / S);
+        const int grid = (int)(niter < (long long)kSMs * stream_ctas<T>() ? niter : (long long)kSMs * stream_ctas<T>());
+        e = launch_k(k_spmv_csr_stream<T>, dim3(grid), dim3(kSThreads), s, rp, col, val, x, y, m, S);
+      } else if (A->variant == 0) {
         // kCsrWarps warps grid-stride over rows (the mapping the csr_max feature describes, Q4); a
         // matrix covered in one pass gets only the warps that own rows (same row -> warp mapping).
         const int tpv = csr_vector_tpv(m, z);
         const long long warps_needed = ceil_div(m, 32 / tpv);
         const int blocks = (int)ceil_div(warps_needed < kCsrWarps ? warps_needed : kCsrWarps, 256 / 32);
         switch (tpv) {
-          case 2: k_spmv_csr_vector<T, 2><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
-          case 4: k_spmv_csr_vector<T, 4><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
-          case 8: k_spmv_csr_vector<T, 8><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
-          case 16: k_spmv_csr_vector<T, 16><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
-          default: k_spmv_csr_vector<T, 32><<<blocks, 256, 0, s>>>(rp, col, val, x, y, m); break;
+          case 2: e = launch_k(k_spmv_csr_vector<T, 2>, dim3(blocks), dim3(256), s, rp, col, val, x, y, m); break;
+          case 4: e = launch_k(k_spmv_csr_vector<T, 4>, dim3(blocks), dim3(256), s, rp, col, val, x, y, m); break;
+          case 8: e = launch_k(k_spmv_csr_vector<T, 8>, dim3(blocks), dim3(256), s, rp, col, val, x, y, m); break;
+          case 16: e = launch_k(k_spmv_csr_vector<T, 16>, dim3(blocks), dim3(256), s, rp, col, val, x, y, m); break;
+          default: e = launch_k(k_spmv_csr_vector<T, 32>, dim3(blocks), dim3(256), s, rp, col, val, x, y, m); break;
         }
-        count_launch();
       } else {
         const long long tiles = ceil_div(m + z, kMTile);
         MergeWork w = merge_work(A->work, tiles);
-        k_spmv_csr_merge<T><<<(unsigned)tiles, kMT, 0, s>>>(rp, col, val, x, y, m, z, w.coords, w.crow, w.cval);
-        k_spmv_csr_merge_fixup<T><<<grid_cap(tiles, 256, 4), 256, 0, s>>>(w.crow, w.cval, tiles, m, y);
-        count_launch(2);
+        e = launch_k(k_spmv_csr_merge<T>, dim3((unsigned)tiles), dim3(kMT), s, rp, col, val, x, y, m, z, w.coords,
+                     w.crow, w.cval);
+        if (e == cudaSuccess)
+          e = launch_k(k_spmv_csr_merge_fixup<T>, dim3(grid_cap(tiles, 256, 4)), dim3(256), s, (const int*)w.crow,
+                       (const acc_t*)w.cval, tiles, m, y);
       }
       break;
     }
     case SFS_COO: {
-      cudaError_t e = cudaMemsetAsync(y, 0, sizeof(T) * m, s);
-      if (e != cudaSuccess) return e;
-      count_launch();
-      if (z > 0) {
-        launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s);
-        count_launch();
-      }
+      e = launch_zero<T>(y, m, s);
+      if (e == cudaSuccess && z > 0)
+        e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s);
       break;
     }
     case SFS_ELL:
     case SFS_HYB: {
       const int K = (int)A->width;
-      if (K == 0) {
-        cudaError_t e = cudaMemsetAsync(y, 0, sizeof(T) * m, s);
-        if (e != cudaSuccess) return e;
-      } else {
-        k_spmv_ell<T><<<grid_cap(A->pitch / 4, kEllThreads, 4), kEllThreads, 0, s>>>(
-            (const int*)A->ptr[0], (const T*)A->ptr[1], x, y, m, A->pitch, K);
-      }
-      count_launch();
-      if (A->fmt == SFS_HYB && A->coo_nnz > 0) {
-        launch_coo<T, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y, A->coo_nnz, s);
-        count_launch();
-      }
+      e = K == 0 ? launch_zero<T>(y, m, s) : launch_ell<T>(A, x, y, K, s);
+      if (e == cudaSuccess && A->fmt == SFS_HYB && A->coo_nnz > 0)
+        e = launch_coo<T, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y, A->coo_nnz, s);
       break;
     }
     case SFS_DIA: {
-      k_spmv_dia<T><<<grid_cap(A->pitch / 4, kDiaThreads, 4), kDiaThreads, 0, s>>>(
-          (const int*)A->ptr[0], (const T*)A->ptr[1], x, y, m, A->n, A->pitch, (int)A->ndiag);
-      count_launch();
+      const long long blocks_rows = ceil_div(m, dia_rows<T>());  // threads needed at S = 1
+      const int S = split_factor(blocks_rows, A->ndiag, 2 * kDiaBatch, 16);
+      const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
+      const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
+      e = launch_k(k_spmv_dia<T>, dim3(grid < 1 ? 1 : grid), dim3(kDiaThreads), s, (const int*)A->ptr[0],
+                   (const T*)A->ptr[1], x, y, m, A->n, A->pitch, (int)A->ndiag, S);
       break;
     }
     default:
       return cudaErrorInvalidValue;
   }
-  return cudaGetLastError();
+  return e;
 }
 
 // Cold-cache mode: stream a 2x-L2 buffer through L2 with plain reads (clean lines, so the next SpMV
@@ -554,7 +802,7 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
-    case SFS_CSR: return A->variant == 0 ? 1 : 2;
+    case SFS_CSR: return A->variant == 1 ? 2 : 1;
     case SFS_COO: return A->nnz > 0 ? 2 : 1;
     case SFS_HYB: return A->coo_nnz > 0 ? 2 : 1;
     default: return 1;

@@ -75,7 +75,7 @@ def test_conversions_bit_exact(name):
 
 
 @pytest.mark.parametrize("name", NAMES)
-@pytest.mark.parametrize("variant", [0, 1])
+@pytest.mark.parametrize("variant", [0, 1, 2])
 def test_spmv_tolerance(name, variant):
     A = cases()[name]
     fo = oracle.features(A.m, A.n, A.rp, A.col)
@@ -85,7 +85,7 @@ def test_spmv_tolerance(name, variant):
     for fmt in range(5):
         if not (fo["admissible_mask"] >> fmt) & 1:
             continue
-        if fmt != sfs.CSR and variant == 1:
+        if fmt != sfs.CSR and variant != 2:
             continue
         M = sfs.convert(dA, fmt, opts)
         check_spmv(A, fmt, M, x, A.dtype, ctx=f"{name}/v{variant}")
@@ -103,9 +103,9 @@ def test_spmv_x_ones_bitwise(dtype, cls, N, pts):
     dA = to_dev(A)
     tdt = torch.float64 if dtype == sfsgen.F64 else torch.float32
     x = torch.ones(A.n, dtype=tdt, device="cuda")
-    for variant in (0, 1):
+    for variant in (0, 1, 2):
         for fmt in range(5):
-            if variant == 1 and fmt != sfs.CSR:
+            if variant != 2 and fmt != sfs.CSR:
                 continue
             M = sfs.convert(dA, fmt, sfs.default_opts(csr_variant=variant))
             y = torch.empty(A.m, dtype=tdt, device="cuda")
