@@ -91,9 +91,9 @@ int split_factor(long long items, long long units, long long per_thread, int sma
 template <typename T>
 __global__ void k_zero(T* __restrict__ y, long long m) {
   pdl_wait();
+  pdl_trigger();  // successor (COO) overlaps its loads with this kernel and waits before storing
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < m; i += (long long)gridDim.x * blockDim.x)
     y[i] = T(0);
-  pdl_trigger();
 }
 
 // ======================================================================== CSR vector
@@ -186,19 +186,22 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
     for (int w0 = s0 + p * kSW; w0 < s1; w0 += S * kSW) {
       const int n = s1 - w0 < kSW ? s1 - w0 : kSW;
       int c[kSU];
-      T v[kSU];
+      T v[kSU], xv[kSU];
+      // Loads are unconditional (indices clamped into the window) so that all 2*kSU of them, then
+      // all kSU x gathers, issue back to back; only the smem stores are predicated.
+      const int last = n - 1;
 #pragma unroll
       for (int u = 0; u < kSU; u++) {
-        const int i = u * 32 + lane;
-        if (i < n) {
-          c[u] = ld_stream(col + w0 + i);
-          v[u] = ld_stream(val + w0 + i);
-        }
+        const int i = u * 32 + lane < n ? u * 32 + lane : last;
+        c[u] = ld_stream(col + w0 + i);
+        v[u] = ld_stream(val + w0 + i);
       }
 #pragma unroll
+      for (int u = 0; u < kSU; u++) xv[u] = ld_x(x + c[u]);
+#pragma unroll
       for (int u = 0; u < kSU; u++) {
         const int i = u * 32 + lane;
-        if (i < n) buf[i] = (acc_t)v[u] * (acc_t)ld_x(x + c[u]);
+        if (i < n) buf[i] = (acc_t)v[u] * (acc_t)xv[u];
       }
       __syncwarp();
       const int lo = (b > w0 ? b : w0) - w0, hi = (e < w0 + n ? e : w0 + n) - w0;
@@ -312,20 +315,24 @@ __global__ void __launch_bounds__(kMT) k_spmv_csr_merge(const int* __restrict__ 
   {
     const int nr = (r1 - r0 + 2 < (int)(m - r0 + 1)) ? r1 - r0 + 2 : (int)(m - r0 + 1);
     const int nk = k1 - k0;
+    // Loads unconditional with clamped (always valid) indices so they all issue back to back; only
+    // the shared-memory stores are predicated.
     int rv[kMI + 1], cv[kMI];
-    T vv[kMI];
+    T vv[kMI], xv[kMI];
 #pragma unroll
     for (int u = 0; u <= kMI; u++) {
       const int i = threadIdx.x + u * kMT;
-      if (i < nr) rv[u] = __ldg(rp + r0 + i);
+      rv[u] = __ldg(rp + r0 + (i < nr ? i : nr - 1));
     }
+    if (nk > 0) {
 #pragma unroll
-    for (int u = 0; u < kMI; u++) {
-      const int i = threadIdx.x + u * kMT;
-      if (i < nk) {
+      for (int u = 0; u < kMI; u++) {
+        const int i = threadIdx.x + u * kMT < nk ? threadIdx.x + u * kMT : nk - 1;
         cv[u] = ld_stream(col + k0 + i);
         vv[u] = ld_stream(val + k0 + i);
       }
+#pragma unroll
+      for (int u = 0; u < kMI; u++) xv[u] = ld_x(x + cv[u]);
     }
 #pragma unroll
     for (int u = 0; u <= kMI; u++) {
@@ -335,7 +342,7 @@ __global__ void __launch_bounds__(kMT) k_spmv_csr_merge(const int* __restrict__ 
 #pragma unroll
     for (int u = 0; u < kMI; u++) {
       const int i = threadIdx.x + u * kMT;
-      if (i < nk) s_prod[i] = (acc_t)vv[u] * (acc_t)ld_x(x + cv[u]);
+      if (i < nk) s_prod[i] = (acc_t)vv[u] * (acc_t)xv[u];
     }
   }
   __syncthreads();
@@ -401,7 +408,9 @@ template <typename T, bool ACCUM>
 __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
                                                           T* __restrict__ y, long long z, long long chunks_per_warp) {
-  pdl_wait();
+  // PDL: the predecessor (zero kernel / ELL part of HYB) released us at its start; everything up to
+  // the first write (or ACCUM read) of y overlaps it.
+  bool waited = false;
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kChunk);
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -442,6 +451,10 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
             p[i] = 0;
           }
         }
+      }
+      if (!waited) {
+        pdl_wait();
+        waited = true;
       }
       const int rf = r[0], rl = r[kCooV - 1];
       // the previous chunk's carry ends exactly at this chunk boundary: emit it
@@ -494,6 +507,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
     }
     if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
   }
+  if (!waited) pdl_wait();
   pdl_trigger();
 }
 
@@ -509,10 +523,12 @@ template <typename T>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
                                                                          const T* __restrict__ eval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
-                                                                         long long m, long long P, int K, int S) {
+                                                                         long long m, long long P, int K, int S,
+                                                                         int early_trigger) {
   constexpr int kB = ell_batch<T>();
   __shared__ acc_t s_part[kEllThreads][4];
   pdl_wait();
+  if (early_trigger) pdl_trigger();  // HYB: let the COO part start its loads now
   const int G = kEllThreads / S;
   const int p = threadIdx.x / G, g = threadIdx.x % G;
   const int Kp = (K + S - 1) / S;
@@ -580,52 +596,77 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
 // loads in flight.  The S diagonal-parts of a row block meet in shared memory.
 constexpr int kDiaThreads = 256;
 constexpr int kDiaSmemOffs = 1024;
-template <typename T> constexpr int dia_rows() { return sizeof(T) == 4 ? 8 : 4; }
-template <typename T> constexpr int dia_ctas() { return sizeof(T) == 4 ? 2 : 3; }  // register cap
-constexpr int kDiaBatch = 4;
+template <typename T> constexpr int dia_rows() { return 4; }
+template <typename T> constexpr int dia_ctas() { return 4; }  // register cap
+template <typename T> constexpr int dia_batch() { return 4; }  // diagonals per batch
 
-template <typename T>
+template <typename T, int S>
 __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const int* __restrict__ offs,
                                                                          const T* __restrict__ dval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
-                                                                         long long m, long long n, long long P, int nd,
-                                                                         int S) {
+                                                                         long long m, long long n, long long P,
+                                                                         int nd) {
   constexpr int kR = dia_rows<T>();
+  constexpr int G = kDiaThreads / S;  // threads per part (compile-time: row strides are immediates)
+  constexpr int kB = dia_batch<T>();
   __shared__ int s_off[kDiaSmemOffs];
-  __shared__ acc_t s_part[kDiaThreads * kR];
+  __shared__ acc_t s_part[S > 1 ? kDiaThreads * kR : 1];
   pdl_wait();
   const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
   for (int i = threadIdx.x; i < nsm; i += blockDim.x) s_off[i] = offs[i];
   __syncthreads();
-  const int G = kDiaThreads / S;
   const int p = threadIdx.x / G, g = threadIdx.x % G;
   const int Dp = (nd + S - 1) / S;
   const int d0 = p * Dp, d1 = d0 + Dp < nd ? d0 + Dp : nd;
-  const long long rows_per_blk = (long long)G * kR;
+  constexpr long long rows_per_blk = (long long)G * kR;
   const long long nblk = ceil_div(m, rows_per_blk);
   for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
-    const long long r0 = blk * rows_per_blk + g;
+    const long long rbase = blk * rows_per_blk;
+    const long long r0 = rbase + g;
+    const bool full = rbase + rows_per_blk <= m;
     acc_t acc[kR];
 #pragma unroll
     for (int q = 0; q < kR; q++) acc[q] = 0;
-    for (int d = d0; d < d1; d += kDiaBatch) {
-      T v[kDiaBatch][kR];
-      int off[kDiaBatch];
+    for (int d = d0; d < d1; d += kB) {
+      const int nb = d1 - d < kB ? d1 - d : kB;
+      int off[kB];
 #pragma unroll
-      for (int u = 0; u < kDiaBatch; u++) {
-        off[u] = d + u < d1 ? (d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u)) : 0;
+      for (int u = 0; u < kB; u++) off[u] = u < nb ? (d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u)) : 0;
+      bool all_in = full && nb == kB;
 #pragma unroll
-        for (int q = 0; q < kR; q++) {
-          const long long rr = r0 + (long long)q * G;
-          v[u][q] = (d + u < d1 && rr < m) ? ld_stream(dval + (long long)(d + u) * P + rr) : T(0);
-        }
+      for (int u = 0; u < kB; u++) {
+        const long long c0 = r0 + off[u];
+        all_in = all_in && c0 >= 0 && c0 + (kR - 1) * G < n;
       }
+      if (all_in) {
+        // fast path (interior blocks): every load unconditional with a per-diagonal base pointer and
+        // immediate row offsets, slab values first, then the x gathers, then the FMAs
+        T v[kB][kR], xv[kB][kR];
 #pragma unroll
-      for (int u = 0; u < kDiaBatch; u++) {
+        for (int u = 0; u < kB; u++) {
+          const T* vp = dval + (long long)(d + u) * P + r0;
 #pragma unroll
-        for (int q = 0; q < kR; q++) {
-          const long long c = r0 + (long long)q * G + (long long)off[u];
-          if (d + u < d1 && c >= 0 && c < n) acc[q] += (acc_t)v[u][q] * (acc_t)ld_x(x + c);
+          for (int q = 0; q < kR; q++) v[u][q] = ld_stream(vp + q * G);
+        }
+#pragma unroll
+        for (int u = 0; u < kB; u++) {
+          const T* xp = x + r0 + off[u];
+#pragma unroll
+          for (int q = 0; q < kR; q++) xv[u][q] = ld_x(xp + q * G);
+        }
+#pragma unroll
+        for (int u = 0; u < kB; u++)
+#pragma unroll
+          for (int q = 0; q < kR; q++) acc[q] += (acc_t)v[u][q] * (acc_t)xv[u][q];
+      } else {
+        for (int u = 0; u < nb; u++) {
+          const T* vp = dval + (long long)(d + u) * P + r0;
+          const long long c0 = r0 + off[u];
+#pragma unroll
+          for (int q = 0; q < kR; q++) {
+            const long long rr = r0 + q * G, c = c0 + q * G;
+            if (rr < m && c >= 0 && c < n) acc[q] += (acc_t)ld_stream(vp + q * G) * (acc_t)ld_x(x + c);
+          }
         }
       }
     }
@@ -634,6 +675,7 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
       for (int q = 0; q < kR; q++) s_part[threadIdx.x * kR + q] = acc[q];
       __syncthreads();
       if (p == 0) {
+#pragma unroll
         for (int pp = 1; pp < S; pp++)
 #pragma unroll
           for (int q = 0; q < kR; q++) acc[q] += s_part[(pp * G + g) * kR + q];
@@ -685,13 +727,13 @@ cudaError_t launch_zero(T* y, long long m, cudaStream_t s) {
 }
 
 template <typename T>
-cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s) {
+cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s, int early_trigger) {
   const long long groups = A->pitch / 4;
   const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
   const long long niter = ceil_div(groups, kEllThreads / S);
   const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
   return launch_k(k_spmv_ell<T>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1], x, y,
-                  A->m, A->pitch, K, S);
+                  A->m, A->pitch, K, S, early_trigger);
 }
 
 template <typename T>
@@ -743,18 +785,27 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
     case SFS_ELL:
     case SFS_HYB: {
       const int K = (int)A->width;
-      e = K == 0 ? launch_zero<T>(y, m, s) : launch_ell<T>(A, x, y, K, s);
+      e = K == 0 ? launch_zero<T>(y, m, s) : launch_ell<T>(A, x, y, K, s, A->fmt == SFS_HYB && A->coo_nnz > 0);
       if (e == cudaSuccess && A->fmt == SFS_HYB && A->coo_nnz > 0)
         e = launch_coo<T, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y, A->coo_nnz, s);
       break;
     }
     case SFS_DIA: {
       const long long blocks_rows = ceil_div(m, dia_rows<T>());  // threads needed at S = 1
-      const int S = split_factor(blocks_rows, A->ndiag, 2 * kDiaBatch, 16);
+      const int S = split_factor(blocks_rows, A->ndiag, 2 * dia_batch<T>(), 16);
       const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
       const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
-      e = launch_k(k_spmv_dia<T>, dim3(grid < 1 ? 1 : grid), dim3(kDiaThreads), s, (const int*)A->ptr[0],
-                   (const T*)A->ptr[1], x, y, m, A->n, A->pitch, (int)A->ndiag, S);
+      const dim3 gd(grid < 1 ? 1 : grid), bd(kDiaThreads);
+      const int* offs = (const int*)A->ptr[0];
+      const T* dv = (const T*)A->ptr[1];
+      const int nd = (int)A->ndiag;
+      switch (S) {
+        case 1: e = launch_k(k_spmv_dia<T, 1>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
+        case 2: e = launch_k(k_spmv_dia<T, 2>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
+        case 4: e = launch_k(k_spmv_dia<T, 4>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
+        case 8: e = launch_k(k_spmv_dia<T, 8>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
+        default: e = launch_k(k_spmv_dia<T, 16>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
+      }
       break;
     }
     default:
