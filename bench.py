@@ -44,6 +44,7 @@ def parse():
     p.add_argument("--corpus", type=int, default=200, help="matrices per rank (configs[1]: 200)")
     p.add_argument("--reps", type=int, default=100)
     p.add_argument("--race-warmup", type=int, default=5)
+    p.add_argument("--graphs", action="store_true", help="capture the timed reps in CUDA graphs")
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--cpu-budget", type=float, default=15.0, help="seconds of oracle work for cpu_baseline")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -222,7 +223,7 @@ def run_ours(args):
     pin = lambda a: torch.from_numpy(a).pin_memory()
     hmats = [sfs.Csr(A.m, A.n, pin(A.rp), pin(A.col), pin(A.val), pin(x)) for _, A, x in host]
     torch.cuda.synchronize()
-    opts = sfs.default_opts(reps=args.reps, warmup=args.race_warmup)
+    opts = sfs.default_opts(reps=args.reps, warmup=args.race_warmup, use_graphs=1 if args.graphs else 0)
     n = len(mats)
     gather_buf = torch.zeros(n * 8, dtype=torch.float64, device=dev)
     all_buf = torch.zeros(world * n * 8, dtype=torch.float64, device=dev)

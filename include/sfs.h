@@ -108,7 +108,7 @@ typedef struct {
   double hyb_rel_speed;  /* Q6 HYB width rule (3.0) */
   int64_t hyb_breakeven; /* (4096) */
   int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream */
-  int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (1) */
+  int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (0: direct launches with PDL) */
 } sfs_race_opts;
 
 /* Result of racing one matrix. */

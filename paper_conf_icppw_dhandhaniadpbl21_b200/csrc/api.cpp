@@ -7,6 +7,9 @@
 
 #include <algorithm>
 #include <atomic>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cmath>
 #include <mutex>
 #include <string>
@@ -109,7 +112,7 @@ static void defaults(sfs_race_opts* o) {
   o->hyb_rel_speed = 3.0;
   o->hyb_breakeven = 4096;
   o->csr_variant = -1;
-  o->use_graphs = 1;
+  o->use_graphs = 0;  // direct PDL launches: measured faster than per-(matrix, format) graphs
 }
 
 // Q6: largest R with  rel * R < m  or  R < breakeven  (the condition is monotone in R).
@@ -605,6 +608,11 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   cudaStream_t s = (cudaStream_t)stream;
   cudaStream_t cap = nullptr;  // capture-only stream (records graphs, executes nothing)
   TRY_CUDA(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
+  cudaStream_t up = nullptr;  // graph uploads (SFS_GRAPH_UPLOAD=0 disables)
+  {
+    const char* eu = getenv("SFS_GRAPH_UPLOAD");
+    if (!(eu && eu[0] == '0')) TRY_CUDA(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
+  }
   EventPool ev;
   std::vector<DevCSR> d(n);
   std::vector<FeatWork> w(n);
@@ -635,6 +643,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   if (e != cudaSuccess) {
     cudaFreeHost(ha);
     cudaStreamDestroy(cap);
+    if (up) cudaStreamDestroy(up);
     return cuda_fail(e, "feature phase");
   }
   for (int64_t i = 0; i < n; i++) {
@@ -642,6 +651,10 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     if (mst[i] == SFS_OK) labels[i].t_features_us = elapsed_us(fe0[i], fe1[i]);
   }
   // ---- phase 2: the race; everything enqueued, no host synchronisation
+  using clk = std::chrono::steady_clock;
+  const bool prof = getenv("SFS_PROFILE") != nullptr;
+  double t_graph = 0, t_inst = 0, t_conv = 0, t_warm = 0;
+  const auto t_phase2 = clk::now();
   struct Timed {
     int64_t i;
     int f;
@@ -696,10 +709,14 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
       T.c1 = ev.get();
       cudaEventRecord(T.c0, s);
       Matrix* A = nullptr;
+      const auto tc0 = clk::now();
       sfs_status st = convert_impl(D, (sfs_format)f, F, w[i], &A, s);
       cudaEventRecord(T.c1, s);
+      const auto tc1 = clk::now();
+      t_conv += std::chrono::duration<double>(tc1 - tc0).count();
       if (st != SFS_OK) { L.status[f] = st; continue; }
       for (int r = 0; r < o.warmup; r++) launch_spmv(A, x, y, s);
+      t_warm += std::chrono::duration<double>(clk::now() - tc1).count();
       const int kpc = spmv_kernels_per_call(A);
       if (o.cold) {
         for (int r = 0; r < o.reps; r++) {
@@ -715,13 +732,24 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
         cudaGraph_t g = nullptr;
         cudaGraphExec_t ge = nullptr;
         const int64_t before = g_launches.load();
+        const auto tg0 = clk::now();
         bool ok = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
         if (ok) {
           for (int r = 0; r < o.reps; r++) launch_spmv(A, x, y, cap);
           ok = cudaStreamEndCapture(cap, &g) == cudaSuccess;
         }
         g_launches.store(before);
+        const auto ti0 = clk::now();
         if (ok) ok = cudaGraphInstantiate(&ge, g, 0) == cudaSuccess;
+        if (ok && up) {
+          // upload the executable graph on a side stream (overlapping the work already queued on s)
+          // instead of paying the implicit upload inside the timed launch
+          cudaEvent_t eu = ev.get();
+          ok = cudaGraphUpload(ge, up) == cudaSuccess && cudaEventRecord(eu, up) == cudaSuccess &&
+               cudaStreamWaitEvent(s, eu, 0) == cudaSuccess;
+        }
+        t_inst += std::chrono::duration<double>(clk::now() - ti0).count();
+        t_graph += std::chrono::duration<double>(clk::now() - tg0).count();
         T.t0 = ev.get();
         T.t1 = ev.get();
         cudaEventRecord(T.t0, s);
@@ -756,10 +784,20 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     unstage(d[i], s);
   }
   if (flush) dfree(flush, s);
+  const auto t_enq = clk::now();
   e = cudaStreamSynchronize(s);
+  if (prof) {
+    const auto t_end = clk::now();
+    fprintf(stderr,
+            "[sfs] label_corpus n=%lld: enqueue %.1f ms (convert %.1f, warmup %.1f, graph capture %.1f + instantiate "
+            "%.1f ms), sync wait %.1f ms\n",
+            (long long)n, 1e3 * std::chrono::duration<double>(t_enq - t_phase2).count(), 1e3 * t_conv, 1e3 * t_warm,
+            1e3 * (t_graph - t_inst), 1e3 * t_inst, 1e3 * std::chrono::duration<double>(t_end - t_enq).count());
+  }
   for (auto ge : execs) cudaGraphExecDestroy(ge);
   for (auto g : graphs) cudaGraphDestroy(g);
   cudaStreamDestroy(cap);
+  if (up) cudaStreamDestroy(up);
   cudaFreeHost(ha);
   if (e != cudaSuccess) return cuda_fail(e, "race");
   for (auto& T : timed) {

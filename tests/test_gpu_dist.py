@@ -1,0 +1,80 @@
+"""Multi-GPU drivers on one GPU: the row partition (configs[3] shape) and the sharded corpus driver
+with the real library (the N > 1 exchange is covered by the gloo tests)."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+import sfsgen
+from gpu_util import TOL
+from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+@pytest.mark.parametrize("fmt", [sfs.CSR, sfs.DIA, sfs.ELL])
+def test_row_partition_blocks_reassemble(world, fmt):
+    """Each rank's row block (global column ids) through sfs_convert / sfs_spmv, x = the full vector
+    (what all_gather_into_tensor delivers), blocks concatenated == oracle y within tolerance."""
+    import torch
+    A = sfsgen.generate(sfsgen.make_spec(sfsgen.ST3D27, ia=24))
+    x = sfsgen.vector(11, A.n)
+    xd = torch.from_numpy(x).cuda()
+    ys = []
+    for rank in range(world):
+        part = sd.RowPartition(A.m, A.n, world, rank)
+        b = part.bounds
+        rp, col, val = sd.slice_rows(A.rp, A.col, A.val, b[rank], b[rank + 1])
+        if part.local_rows == 0:
+            continue
+        t = lambda a: torch.from_numpy(a).cuda()
+        Ak = sfs.Csr(part.local_rows, A.n, t(rp), t(col), t(val))
+        M = sfs.convert(Ak, fmt)
+        y = torch.empty(part.local_rows, dtype=torch.float64, device="cuda")
+        sfs.spmv(fmt, M, xd, y)
+        ys.append(y.cpu().numpy())
+        M.free()
+    y = np.concatenate(ys)
+    yr, ay = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
+    assert np.all(np.abs(y - yr) <= TOL[sfs.F64] * ay)
+
+
+def test_rowpart_iterate_single_rank_power_iteration():
+    import torch
+    A = sfsgen.generate(sfsgen.make_spec(sfsgen.ST2D5, ia=40))
+    part = sd.RowPartition(A.m, A.n, 1, 0)
+    t = lambda a: torch.from_numpy(a).cuda()
+    M = sfs.convert(sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val)), sfs.CSR)
+    x0 = sfsgen.vector(3, A.n)
+    y = sd.rowpart_spmv_iterate(part, lambda xf, yl: sfs.spmv(sfs.CSR, M, xf, yl), t(x0), iters=3)
+    xr = x0
+    for _ in range(3):
+        xr, _ = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, xr)
+    assert np.allclose(y.cpu().numpy(), xr, rtol=1e-11, atol=1e-12)
+
+
+def test_sharded_corpus_driver_single_rank():
+    import torch
+    ids = list(range(6))
+
+    def make(i):
+        A = sfsgen.generate(sfsgen.make_spec(sfsgen.BAND if i % 2 else sfsgen.UNIFORM, seed=i + 3, m=2000 + 100 * i,
+                                             ia=4, pa=9.0))
+        t = lambda a: torch.from_numpy(a).cuda()
+        return sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val)), A
+
+    cache = {}
+
+    def mk(i):
+        cache[i] = make(i)
+        return cache[i][0]
+
+    res = sd.label_corpus_sharded(ids, [1.0] * len(ids), mk, lambda b: sfs.label_corpus(b, sfs.default_opts(reps=5)),
+                                  rank=0, world=1, batch_bytes=1e5, nbytes=lambda m: m.nbytes())
+    assert [r["id"] for r in res] == ids
+    for r in res:
+        A = cache[r["id"]][1]
+        fo = oracle.features(A.m, A.n, A.rp, A.col)
+        assert r["features"]["nnz"] == fo["nnz"] and r["features"]["nnz_sig"] == fo["nnz_sig"]
+        assert 0 <= r["label"] < 5 and r["matrix_status"] == 0
