@@ -167,7 +167,7 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
                                                                T* __restrict__ y, long long m, int S) {
   constexpr int kSU = stream_u<T>();  // all of a lane's loads of a window are in flight together
   constexpr int kSW = 32 * kSU;
-  __shared__ acc_t sbuf[kSWarps][kSWMax];
+  __shared__ acc_t sbuf[kSWarps][kSW];
   __shared__ acc_t s_part[kSWarps][32];
   pdl_wait();
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
@@ -176,11 +176,21 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
   acc_t* buf = sbuf[w];
   const long long ngroups = ceil_div(m, 32);
   const long long niter = ceil_div(ngroups, NG);
+  // row bounds of the group are prefetched one iteration ahead (off the col -> x critical path)
+  auto bounds = [&](long long it, int& b, int& e) {
+    const long long g = it * NG + gl;
+    const long long r = g * 32 + lane;
+    const long long rb = g < ngroups ? (r < m ? r : m) : m;
+    b = __ldg(rp + rb);
+    e = __ldg(rp + (g < ngroups && r < m ? r + 1 : rb));
+  };
+  int nb = 0, ne = 0;
+  if ((long long)blockIdx.x < niter) bounds(blockIdx.x, nb, ne);
   for (long long it = blockIdx.x; it < niter; it += gridDim.x) {
     const long long g = it * NG + gl;
     const long long r = g * 32 + lane;
-    const int b = g < ngroups ? __ldg(rp + (r < m ? r : m)) : 0;
-    const int e = g < ngroups ? __ldg(rp + (r < m ? r + 1 : m)) : 0;
+    const int b = nb, e = ne;
+    if (it + gridDim.x < niter) bounds(it + gridDim.x, nb, ne);
     const int s0 = __shfl_sync(0xffffffffu, b, 0), s1 = __shfl_sync(0xffffffffu, e, 31);
     acc_t acc = 0;
     for (int w0 = s0 + p * kSW; w0 < s1; w0 += S * kSW) {

@@ -31,8 +31,8 @@ def make_matrix(name):
         return sfsgen.stencil3d27(128, dtype=sfsgen.F32)
     if name == "laplace64":
         return sfsgen.laplace2d(64)
-    if name.startswith("corpus:"):
-        return sfsgen.generate(sfsgen.corpus_spec(200, int(name.split(":")[1])))
+    if name.startswith("corpus:") or name.startswith("corpus-"):
+        return sfsgen.generate(sfsgen.corpus_spec(200, int(name[7:])))
     if name == "band_big":
         return sfsgen.generate(sfsgen.make_spec(sfsgen.BAND, seed=11, m=1_000_000, ia=24, pa=0.8))
     if name == "uniform_big":
