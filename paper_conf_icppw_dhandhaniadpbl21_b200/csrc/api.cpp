@@ -626,10 +626,22 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     labels[i].label = -1;
     for (int f = 0; f < SFS_NFMT; f++) labels[i].status[f] = SFS_ERR_NOT_RUN;
   }
+  cudaStream_t cs = nullptr;  // H2D copy stream for host-memory inputs
+  for (int64_t i = 0; i < n; i++)
+    if (mats[i].mem == SFS_MEM_HOST) {
+      TRY_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+      break;
+    }
   // ---- phase 1: stage + features of every matrix, one synchronisation
   for (int64_t i = 0; i < n; i++) {
     sfs_status st = check_csr(&mats[i]);
-    if (st == SFS_OK) st = stage(&mats[i], d[i], s, true);
+    // host inputs: stage on the copy stream so the H2D of matrix i+1 overlaps the features of i
+    if (st == SFS_OK) st = stage(&mats[i], d[i], cs ? cs : s, true);
+    if (st == SFS_OK && d[i].host && cs) {
+      cudaEvent_t ec = ev.get();
+      cudaEventRecord(ec, cs);
+      cudaStreamWaitEvent(s, ec, 0);
+    }
     if (st == SFS_OK) {
       fe0[i] = ev.get();
       fe1[i] = ev.get();
@@ -644,6 +656,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     cudaFreeHost(ha);
     cudaStreamDestroy(cap);
     if (up) cudaStreamDestroy(up);
+    if (cs) cudaStreamDestroy(cs);
     return cuda_fail(e, "feature phase");
   }
   for (int64_t i = 0; i < n; i++) {
@@ -798,6 +811,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   for (auto g : graphs) cudaGraphDestroy(g);
   cudaStreamDestroy(cap);
   if (up) cudaStreamDestroy(up);
+  if (cs) cudaStreamDestroy(cs);
   cudaFreeHost(ha);
   if (e != cudaSuccess) return cuda_fail(e, "race");
   for (auto& T : timed) {
