@@ -53,18 +53,18 @@ def build_oracle(force=False):
     return out
 
 
-def build_sfs(force=False, verbose=False):
+def build_sfs(force=False, verbose=False, variant="", defines=()):
     cu = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
     cpp = sorted(glob.glob(os.path.join(CSRC, "*.cpp")))
     hdr = sorted(glob.glob(os.path.join(CSRC, "*.cuh")) + glob.glob(os.path.join(CSRC, "*.h"))
                  + glob.glob(os.path.join(ROOT, "include", "*.h")))
-    out = os.path.join(PKG, "libsfs.so")
+    out = os.path.join(PKG, f"libsfs{variant}.so")
     if not (force or _stale(out, cu + cpp + hdr)):
         return out
-    objdir = os.path.join(ROOT, "build", "obj")
+    objdir = os.path.join(ROOT, "build", "obj" + variant)
     os.makedirs(objdir, exist_ok=True)
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
-    common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-lineinfo"] + inc
+    common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-lineinfo"] + inc + [f"-D{d}" for d in defines]
 
     def compile_one(src):
         obj = os.path.join(objdir, os.path.basename(src) + ".o")

@@ -13,7 +13,7 @@ from dataclasses import dataclass, field
 from typing import List, Optional, Sequence
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libsfs.so")
+LIB_PATH = os.environ.get("SFS_LIB") or os.path.join(_HERE, "libsfs.so")  # SFS_LIB: A/B builds
 
 CSR, COO, ELL, HYB, DIA = range(5)
 NFMT = 5

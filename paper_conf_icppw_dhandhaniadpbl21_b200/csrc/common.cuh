@@ -9,39 +9,91 @@ namespace sfs {
 
 
 // ---------------------------------------------------------------- cache-hinted loads
-// A's arrays are streamed once per SpMV: no L1 allocation (they would only evict x).
+// A's arrays are streamed once per SpMV: no L1 allocation (they would only evict x).  With
+// SFS_STREAM_EVICT_FIRST the streams also carry an L2 evict-first cache policy (createpolicy +
+// .L2::cache_hint), so that a matrix larger than L2 does not push x out of it.
+#ifdef SFS_STREAM_EVICT_FIRST
+#define SFS_LDS(TY, ...)                                                                              \
+  asm("{\n .reg .b64 pol;\n createpolicy.fractional.L2::evict_first.b64 pol, 1.0;\n"                    \
+      " ld.global.nc.L1::no_allocate.L2::cache_hint" TY ";\n}" : __VA_ARGS__)
+#else
+#define SFS_LDS(TY, ...) asm("ld.global.nc.L1::no_allocate" TY ";" : __VA_ARGS__)
+#endif
 __device__ __forceinline__ int ld_stream(const int* p) {
   int v;
-  asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));
+#ifdef SFS_STREAM_EVICT_FIRST
+  SFS_LDS(".b32 %0, [%1], pol", "=r"(v) : "l"(p));
+#else
+  SFS_LDS(".b32 %0, [%1]", "=r"(v) : "l"(p));
+#endif
   return v;
 }
 __device__ __forceinline__ float ld_stream(const float* p) {
   float v;
-  asm("ld.global.nc.L1::no_allocate.f32 %0, [%1];" : "=f"(v) : "l"(p));
+#ifdef SFS_STREAM_EVICT_FIRST
+  SFS_LDS(".f32 %0, [%1], pol", "=f"(v) : "l"(p));
+#else
+  SFS_LDS(".f32 %0, [%1]", "=f"(v) : "l"(p));
+#endif
   return v;
 }
 __device__ __forceinline__ double ld_stream(const double* p) {
   double v;
-  asm("ld.global.nc.L1::no_allocate.f64 %0, [%1];" : "=d"(v) : "l"(p));
+#ifdef SFS_STREAM_EVICT_FIRST
+  SFS_LDS(".f64 %0, [%1], pol", "=d"(v) : "l"(p));
+#else
+  SFS_LDS(".f64 %0, [%1]", "=d"(v) : "l"(p));
+#endif
   return v;
 }
 __device__ __forceinline__ int4 ld_stream4(const int* p) {
   int4 v;
-  asm("ld.global.nc.L1::no_allocate.v4.s32 {%0,%1,%2,%3}, [%4];"
-               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+#ifdef SFS_STREAM_EVICT_FIRST
+  SFS_LDS(".v4.s32 {%0,%1,%2,%3}, [%4], pol", "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+#else
+  SFS_LDS(".v4.s32 {%0,%1,%2,%3}, [%4]", "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+#endif
   return v;
 }
 __device__ __forceinline__ float4 ld_stream4(const float* p) {
   float4 v;
-  asm("ld.global.nc.L1::no_allocate.v4.f32 {%0,%1,%2,%3}, [%4];"
-               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+#ifdef SFS_STREAM_EVICT_FIRST
+  SFS_LDS(".v4.f32 {%0,%1,%2,%3}, [%4], pol", "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+#else
+  SFS_LDS(".v4.f32 {%0,%1,%2,%3}, [%4]", "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+#endif
   return v;
 }
 __device__ __forceinline__ double2 ld_stream2(const double* p) {
   double2 v;
-  asm("ld.global.nc.L1::no_allocate.v2.f64 {%0,%1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
+#ifdef SFS_STREAM_EVICT_FIRST
+  SFS_LDS(".v2.f64 {%0,%1}, [%2], pol", "=d"(v.x), "=d"(v.y) : "l"(p));
+#else
+  SFS_LDS(".v2.f64 {%0,%1}, [%2]", "=d"(v.x), "=d"(v.y) : "l"(p));
+#endif
   return v;
 }
+// 256-bit streaming loads (sm_100: LDG.E.NA.ENL2.256), 32-byte aligned addresses.
+__device__ __forceinline__ void ld_stream8(const int* p, int (&v)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+      : "l"(p));
+}
+__device__ __forceinline__ void ld_stream8(const float* p, float (&v)[8]) {
+  asm("ld.global.nc.L1::no_allocate.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=f"(v[0]), "=f"(v[1]), "=f"(v[2]), "=f"(v[3]), "=f"(v[4]), "=f"(v[5]), "=f"(v[6]), "=f"(v[7])
+      : "l"(p));
+}
+__device__ __forceinline__ void ld_stream4d(const double* p, double* v) {
+  asm("ld.global.nc.L1::no_allocate.v4.f64 {%0,%1,%2,%3}, [%4];"
+      : "=d"(v[0]), "=d"(v[1]), "=d"(v[2]), "=d"(v[3])
+      : "l"(p));
+}
+__device__ __forceinline__ void ld_stream8(const double* p, double (&v)[8]) {
+  ld_stream4d(p, v);
+  ld_stream4d(p + 4, v + 4);
+}
+
 // x is gathered: keep it in L1 / L2 (read-only path).
 template <typename T>
 __device__ __forceinline__ T ld_x(const T* p) { return __ldg(p); }
@@ -61,10 +113,7 @@ template <> struct Vec4<float> {
 };
 template <> struct Vec4<double> {
   double v[4];
-  __device__ __forceinline__ void load_stream(const double* p) {
-    double2 a = ld_stream2(p), b = ld_stream2(p + 2);
-    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
-  }
+  __device__ __forceinline__ void load_stream(const double* p) { ld_stream4d(p, v); }  // one 256-bit load
   __device__ __forceinline__ void load_x(const double* p) {  // 16 B aligned, cached
     double2 a = __ldg((const double2*)p), b = __ldg((const double2*)p + 1);
     v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
