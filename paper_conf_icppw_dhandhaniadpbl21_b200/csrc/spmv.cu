@@ -160,14 +160,11 @@ template <typename T> constexpr int stream_u() { return sizeof(T) == 4 ? 16 : 8;
 template <typename T> constexpr int stream_ctas() { return sizeof(T) == 4 ? 3 : 4; }  // register cap
 constexpr int kSWMax = 32 * 16;
 
-// VEC: windows start 8-aligned and lane l loads its kSU contiguous items with 256-bit loads (col,
-// val 32 B aligned); products go to smem transposed (item i of the window at (i % kSU) * 32 + i / kSU)
-// so the stores are bank-conflict free.  !VEC: lane l loads items l, l+32, ... (any alignment).
-template <typename T, bool VEC>
+template <typename T>
 __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream(const int* __restrict__ rp,
                                                                const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
-                                                               T* __restrict__ y, long long m, long long z, int S) {
+                                                               T* __restrict__ y, long long m, int S) {
   constexpr int kSU = stream_u<T>();  // all of a lane's loads of a window are in flight together
   constexpr int kSW = 32 * kSU;
   __shared__ acc_t sbuf[kSWarps][kSW];
@@ -196,58 +193,35 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
     if (it + gridDim.x < niter) bounds(it + gridDim.x, nb, ne);
     const int s0 = __shfl_sync(0xffffffffu, b, 0), s1 = __shfl_sync(0xffffffffu, e, 31);
     acc_t acc = 0;
-    const int wbase = VEC ? (s0 & ~7) : s0;
-    for (int w0 = wbase + p * kSW; w0 < s1; w0 += S * kSW) {
+    for (int w0 = s0 + p * kSW; w0 < s1; w0 += S * kSW) {
       const int n = s1 - w0 < kSW ? s1 - w0 : kSW;
-      if (VEC && (long long)w0 + kSW <= z) {
-        // 256-bit path: lane owns items [w0 + lane*kSU, +kSU); items outside [s0, s1) are loaded
-        // (valid columns of the neighbouring rows) but never summed
-        int c[kSU];
-        T v[kSU], xv[kSU];
+      int c[kSU];
+      T v[kSU], xv[kSU];
+      // Loads are unconditional (indices clamped into the window) so that all 2*kSU of them, then
+      // all kSU x gathers, issue back to back; only the smem stores are predicated.
+      const int last = n - 1;
 #pragma unroll
-        for (int h = 0; h < kSU / 8; h++) {
-          int ch[8];
-          T vh[8];
-          ld_stream8(col + w0 + lane * kSU + 8 * h, ch);
-          ld_stream8(val + w0 + lane * kSU + 8 * h, vh);
+      for (int u = 0; u < kSU; u++) {
+        const int i = u * 32 + lane < n ? u * 32 + lane : last;
+        c[u] = ld_stream(col + w0 + i);
+        v[u] = ld_stream(val + w0 + i);
+      }
 #pragma unroll
-          for (int u = 0; u < 8; u++) { c[8 * h + u] = ch[u]; v[8 * h + u] = vh[u]; }
-        }
+      for (int u = 0; u < kSU; u++) xv[u] = ld_x(x + c[u]);
 #pragma unroll
-        for (int u = 0; u < kSU; u++) xv[u] = ld_x(x + c[u]);
-#pragma unroll
-        for (int u = 0; u < kSU; u++) buf[u * 32 + lane] = (acc_t)v[u] * (acc_t)xv[u];
-      } else {
-        // Loads are unconditional (indices clamped into the window) so that all 2*kSU of them, then
-        // all kSU x gathers, issue back to back; only the smem stores are predicated.
-        int c[kSU];
-        T v[kSU], xv[kSU];
-        const int last = n - 1;
-#pragma unroll
-        for (int u = 0; u < kSU; u++) {
-          const int i = VEC ? lane * kSU + u : u * 32 + lane;
-          const int ic = i < n ? i : last;
-          c[u] = ld_stream(col + w0 + ic);
-          v[u] = ld_stream(val + w0 + ic);
-        }
-#pragma unroll
-        for (int u = 0; u < kSU; u++) xv[u] = ld_x(x + c[u]);
-#pragma unroll
-        for (int u = 0; u < kSU; u++) {
-          const int i = VEC ? lane * kSU + u : u * 32 + lane;
-          if (i < n) buf[u * 32 + lane] = (acc_t)v[u] * (acc_t)xv[u];
-        }
+      for (int u = 0; u < kSU; u++) {
+        const int i = u * 32 + lane;
+        if (i < n) buf[i] = (acc_t)v[u] * (acc_t)xv[u];
       }
       __syncwarp();
-      // window item i lives at smem slot  VEC: (i % kSU) * 32 + i / kSU ;  !VEC: i
       const int lo = (b > w0 ? b : w0) - w0, hi = (e < w0 + n ? e : w0 + n) - w0;
       acc_t a0 = 0, a1 = 0;
       int i = lo;
       for (; i + 1 < hi; i += 2) {
-        a0 += buf[VEC ? (i % kSU) * 32 + i / kSU : i];
-        a1 += buf[VEC ? ((i + 1) % kSU) * 32 + (i + 1) / kSU : i + 1];
+        a0 += buf[i];
+        a1 += buf[i + 1];
       }
-      if (i < hi) a0 += buf[VEC ? (i % kSU) * 32 + i / kSU : i];
+      if (i < hi) a0 += buf[i];
       acc += a0 + a1;
       __syncwarp();
     }
@@ -781,11 +755,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
         const long long niter = ceil_div(groups, kSWarps / S);
         const int grid = (int)(niter < (long long)kSMs * stream_ctas<T>() ? niter : (long long)kSMs * stream_ctas<T>());
-        const bool vec = ((uintptr_t)col % 32 == 0) && ((uintptr_t)val % 32 == 0);
-        if (vec)
-          e = launch_k(k_spmv_csr_stream<T, true>, dim3(grid), dim3(kSThreads), s, rp, col, val, x, y, m, z, S);
-        else
-          e = launch_k(k_spmv_csr_stream<T, false>, dim3(grid), dim3(kSThreads), s, rp, col, val, x, y, m, z, S);
+        e = launch_k(k_spmv_csr_stream<T>, dim3(grid), dim3(kSThreads), s, rp, col, val, x, y, m, S);
       } else if (A->variant == 0) {
         // kCsrWarps warps grid-stride over rows (the mapping the csr_max feature describes, Q4); a
         // matrix covered in one pass gets only the warps that own rows (same row -> warp mapping).
