@@ -46,10 +46,10 @@ def build_gen(force=False):
 
 
 def build_oracle(force=False):
-    src = [os.path.join(ROOT, "oracle", "oracle.c"), os.path.join(ROOT, "oracle", "oracle.h")]
+    src = [os.path.join(ROOT, "oracle", f) for f in ("oracle.c", "semisup.c", "oracle.h")]
     out = os.path.join(ROOT, "oracle", "liboracle.so")
     if force or _stale(out, src):
-        _run(["gcc", "-O2", "-std=gnu11", "-fPIC", "-shared", src[0], "-o", out, "-lm"])
+        _run(["gcc", "-O2", "-std=gnu11", "-ffp-contract=off", "-fPIC", "-shared", src[0], src[1], "-o", out, "-lm"])
     return out
 
 

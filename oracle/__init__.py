@@ -207,3 +207,112 @@ def label_matrix(m, n, rp, col, val, x, reps=3, formats_mask=0x1F, opts: Opts | 
     lab = lib().or_label_matrix(m, n, _p(rp), _p(col), _p(val), _p(x), ctypes.byref(opts or default_opts()),
                                 reps, formats_mask, ctypes.byref(f), _p(ts), _p(tc))
     return int(lab), f.as_dict(), ts, tc
+
+
+# ---------------------------------------------------------------------------- semi-supervised (f1)
+# Oracle of the paper's semi-supervised predictor (§4): transform + min-max +
+# PCA(8) + K-Means + VOTE; see oracle/semisup.c and DESIGN.md readings F1–F7.
+NFEAT = 21
+TABLE1 = ["nrows", "ncols", "nnz", "nnz_frac", "nnz_mu", "nnz_min", "nnz_max", "nnz_sig", "max_mu", "mu_min",
+          "csr_max", "sig_lower", "sig_higher", "hyb_ell_size", "hyb_coo", "hyb_ell_frac", "diagonals", "dia_size",
+          "dia_frac", "ell_frac", "ell_size"]
+_ss_ready = False
+
+
+def _ss():
+    global _ss_ready
+    L = lib()
+    if not _ss_ready:
+        L.or_ss_preprocess.argtypes = [_I64, _P, _P, _P, _P]
+        L.or_ss_pca.argtypes = [_I64, ctypes.c_int, _P, ctypes.c_int, _P, _P, _P]
+        L.or_ss_project.argtypes = [_I64, ctypes.c_int, _P, _P, ctypes.c_int, _P, _P]
+        L.or_ss_assign.argtypes = [_I64, ctypes.c_int, _P, ctypes.c_int, _P, _P]
+        L.or_ss_kmeans.argtypes = [_I64, ctypes.c_int, _P, ctypes.c_int, _P, ctypes.c_int, _P, _P]
+        L.or_ss_kmeans.restype = ctypes.c_int
+        L.or_ss_vote.argtypes = [_I64, _P, _P, ctypes.c_int, ctypes.c_int, _P]
+        L.or_ss_purity.argtypes = [_I64, _P, _P, ctypes.c_int, ctypes.c_int, _P]
+        L.or_ss_purity.restype = ctypes.c_double
+        L.or_ss_vote_expected_accuracy.argtypes = [_P, ctypes.c_int, ctypes.c_int, _P]
+        L.or_ss_vote_expected_accuracy.restype = ctypes.c_double
+        L.or_ss_feature_kind.argtypes = [ctypes.c_int]
+        L.or_ss_feature_kind.restype = ctypes.c_int
+        _ss_ready = True
+    return L
+
+
+def table1_matrix(feature_dicts) -> np.ndarray:
+    """n x 21 fp64 matrix of the Table-1 features (P:L79–102 order)."""
+    return np.array([[float(f[k]) for k in TABLE1] for f in feature_dicts], dtype=np.float64).reshape(-1, NFEAT)
+
+
+def ss_preprocess(raw):
+    """F1 transform (log1p / sqrt per feature kind) + F2 min-max to [0, 1]."""
+    raw = _f64(raw).reshape(-1, NFEAT)
+    n = raw.shape[0]
+    out = np.empty_like(raw)
+    mins, maxs = np.empty(NFEAT), np.empty(NFEAT)
+    _ss().or_ss_preprocess(n, _p(raw), _p(out), _p(mins), _p(maxs))
+    return out, mins, maxs
+
+
+def ss_pca(X, k=8):
+    """F3: population covariance, cyclic Jacobi, descending eigenvalues, sign-normalised."""
+    X = _f64(X)
+    n, d = X.shape
+    mean, basis, ev = np.empty(d), np.empty((k, d)), np.empty(k)
+    _ss().or_ss_pca(n, d, _p(X), k, _p(mean), _p(basis), _p(ev))
+    return mean, basis, ev
+
+
+def ss_project(X, mean, basis):
+    X = _f64(X)
+    n, d = X.shape
+    k = basis.shape[0]
+    Y = np.empty((n, k))
+    _ss().or_ss_project(n, d, _p(X), _p(_f64(mean)), k, _p(_f64(basis)), _p(Y))
+    return Y
+
+
+def ss_kmeans(Y, init_idx, max_iter=100):
+    """F4: Lloyd's K-Means from the given initial points."""
+    Y = _f64(Y)
+    n, k = Y.shape
+    init = _i32(init_idx)
+    nc = len(init)
+    cent = np.empty((nc, k))
+    assign = np.empty(n, np.int32)
+    it = _ss().or_ss_kmeans(n, k, _p(Y), nc, _p(init), max_iter, _p(cent), _p(assign))
+    return cent, assign, int(it)
+
+
+def ss_assign(Y, cent):
+    """Nearest centroid, ties to the lowest id."""
+    Y, cent = _f64(Y), _f64(cent)
+    n, k = Y.shape
+    assign = np.empty(n, np.int32)
+    _ss().or_ss_assign(n, k, _p(Y), cent.shape[0], _p(cent), _p(assign))
+    return assign
+
+
+def ss_vote(assign, labels, nc, nfmt=NFMT):
+    """F5/F6: majority of benchmarked members (labels < 0 = not benchmarked)."""
+    a, lab = _i32(assign), _i32(labels)
+    out = np.empty(nc, np.int32)
+    _ss().or_ss_vote(len(a), _p(a), _p(lab), nc, nfmt, _p(out))
+    return out
+
+
+def ss_purity(assign, labels, nc, nfmt=NFMT):
+    """P:L140 purity per cluster and the size-weighted mean."""
+    a, lab = _i32(assign), _i32(labels)
+    pur = np.empty(nc)
+    mean = _ss().or_ss_purity(len(a), _p(a), _p(lab), nc, nfmt, _p(pur))
+    return pur, float(mean)
+
+
+def ss_vote_expected_accuracy(counts, draws):
+    """P:L169 worked example: expected accuracy of a cluster labelled by `draws` benchmarked members."""
+    c = np.ascontiguousarray(counts, dtype=np.int64)
+    p = np.empty(len(c))
+    acc = _ss().or_ss_vote_expected_accuracy(_p(c), len(c), draws, _p(p))
+    return float(acc), p
