@@ -326,22 +326,34 @@ def run_ours(args):
     peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
     if not peak:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
-    traffic = None
+    kernels = {"CSR": "k_spmv_csr_stream (regular rows) / k_spmv_csr_merge + fixup (skewed rows)",
+               "COO": "k_zero + k_spmv_coo", "ELL": "k_spmv_ell", "HYB": "k_spmv_ell + k_spmv_coo<ACCUM>",
+               "DIA": "k_spmv_dia"}
+    achieved = per_fmt[dom]["gbs"]
+    launches_dom = sum(1 for L in labs if L["status"][sfs.FORMAT_NAMES.index(dom)] == 0) * args.reps
+    bytes_per_launch = (per_fmt[dom]["gbs"] * 1e9 * per_fmt[dom]["spmv_time_s"] / launches_dom) if launches_dom else 0
+    traffic, traffic_src = None, None
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
-            traffic = json.load(fh).get(dom)
+            tj = json.load(fh).get(dom)
+        if tj:  # measured DRAM/algorithmic ratio of this format's kernel (ncu --set full, cold, configs[3])
+            traffic = tj["ratio"] * bytes_per_launch
+            traffic_src = (f"dram__bytes_read+write / algorithmic = {tj['ratio']:.3f} for {tj['kernel']} "
+                           f"(profiles/traffic.json), times the mean algorithmic bytes per launch")
     except Exception:
         pass
-    achieved = per_fmt[dom]["gbs"]
     step_time = t_dev / args.steps
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak if achieved else None, "traffic": traffic,
-                "kernel": f"SpMV {dom} ({'k_spmv_csr_vector / k_spmv_csr_merge' if dom == 'CSR' else 'k_spmv_' + dom.lower()})",
-                "peak_source": peak_src,
+                "frac": achieved / peak if achieved else None, "traffic": traffic, "traffic_source": traffic_src,
+                "kernel": f"SpMV {dom}: {kernels[dom]}", "bytes_per_launch": bytes_per_launch,
+                "launches": launches_dom, "peak_source": peak_src,
                 "share_of_step": per_fmt[dom]["spmv_time_s"] / step_time,
-                "note": "achieved = sum over matrices of algorithmic bytes (SURVEY 8(a) a9-a13) x reps / sum of "
-                        "event-timed race time; hot back-to-back reps (P:L217), so matrices that fit in L2 count at "
-                        "L2 speed; gbs_footprint_gt_2xL2 in per_format restricts to footprints > 256 MB"}
+                "achieved_footprint_gt_2xL2": per_fmt[dom]["gbs_footprint_gt_2xL2"],
+                "note": "achieved = sum over the step's matrices of algorithmic bytes (SURVEY 8(a) a9-a13) x reps / "
+                        "sum of their event-timed race time (CUDA events on the launching stream); reps run "
+                        "back-to-back (P:L217), so the many corpus matrices that fit the 126 MB L2 are latency- "
+                        "and L2-bound rather than HBM-bound; achieved_footprint_gt_2xL2 restricts to footprints "
+                        "> 256 MB"}
 
     # ---- CPU oracle baseline (rank 0, N = 1 only)
     cpu = None

@@ -64,7 +64,7 @@ def build_sfs(force=False, verbose=False, variant="", defines=()):
     objdir = os.path.join(ROOT, "build", "obj" + variant)
     os.makedirs(objdir, exist_ok=True)
     inc = ["-I", os.path.join(ROOT, "include"), "-I", CSRC]
-    common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "-lineinfo"] + inc + [f"-D{d}" for d in defines]
+    common = ["-O3", "-std=c++17", "-Xcompiler", "-fPIC,-O3,-ffp-contract=off", "-lineinfo"] + inc + [f"-D{d}" for d in defines]
 
     def compile_one(src):
         obj = os.path.join(objdir, os.path.basename(src) + ".o")

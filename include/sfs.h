@@ -171,6 +171,44 @@ void sfs_set_allocator(void *(*alloc)(size_t bytes, void *stream), void (*deallo
    Lets benchmarks state how many of *our* kernels ran inside a timed region. */
 int64_t sfs_launch_count(void);
 
+/* ---------------------------------------------------------------------------------------------
+ * Semi-supervised format predictor (§4), fitted on the
+ * Table-1 features of a labelled corpus: log1p / sqrt transform and min-max scaling, PCA to
+ * `pcs` components, K-Means with `nc` clusters, cluster label = majority
+ * vote of the benchmarked members, prediction = label of the nearest centroid.
+ * Readings F1–F7 (transform per feature, PCA sign, K-Means start / stop, vote ties): DESIGN.md.
+ * All arrays are HOST arrays (the data is small); the corpus-sized work runs on the GPU.  Syncs. */
+#define SFS_NFEAT 21
+typedef struct {
+  int32_t nc;       /* clusters */
+  int32_t pcs;      /* PCA components (8; <= 16) */
+  int32_t max_iter; /* K-Means iteration cap (100); stops early when no assignment changes */
+} sfs_cluster_opts;
+typedef struct sfs_cluster_model_ *sfs_cluster_model;
+typedef struct {
+  int64_t n;                 /* training matrices */
+  int32_t nc, pcs, iters;
+  const int32_t *assign;     /* n: cluster of every training matrix */
+  const double *centroids;   /* nc x pcs */
+  const double *basis;       /* pcs x 21 (row = component) */
+  const double *eigval;      /* pcs */
+  const double *mins, *maxs; /* 21: transformed-feature ranges used for scaling */
+  const double *mean;        /* 21: mean of the scaled training features */
+} sfs_cluster_info;
+
+/* n x 21 Table-1 matrix (P:L79–102 order) from feature records (host in, host out). */
+sfs_status sfs_features_table1(const sfs_features_t *f, int64_t n, double *out);
+/* Fit on n matrices (table1: n x 21 host).  init_idx: nc distinct indices of the starting points
+   (drawn by the caller, e.g. from a seeded generator).  INVALID_ARG on bad sizes / indices. */
+sfs_status sfs_cluster_fit(const double *table1, int64_t n, const int32_t *init_idx, const sfs_cluster_opts *opt,
+                           sfs_cluster_model *out, void *stream);
+/* labels: n formats of the training matrices, -1 = not benchmarked; cluster_label: nc (host). */
+sfs_status sfs_cluster_vote(sfs_cluster_model M, const int32_t *labels, int32_t *cluster_label, void *stream);
+/* Nearest-centroid cluster of q new matrices (table1: q x 21 host) -> cluster (q, host). */
+sfs_status sfs_cluster_predict(sfs_cluster_model M, const double *table1, int64_t q, int32_t *cluster, void *stream);
+sfs_status sfs_cluster_describe(sfs_cluster_model M, sfs_cluster_info *out);
+sfs_status sfs_cluster_free(sfs_cluster_model M);
+
 /* Library version string. */
 const char *sfs_version(void);
 

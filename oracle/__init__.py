@@ -316,3 +316,28 @@ def ss_vote_expected_accuracy(counts, draws):
     p = np.empty(len(c))
     acc = _ss().or_ss_vote_expected_accuracy(_p(c), len(c), draws, _p(p))
     return float(acc), p
+
+
+def ss_scale(raw, mins, maxs):
+    """Prediction-path scaling of new matrices with the fitted ranges (F2)."""
+    raw = _f64(raw).reshape(-1, NFEAT)
+    out = np.empty_like(raw)
+    L = _ss()
+    L.or_ss_scale.argtypes = [_I64, _P, _P, _P, _P]
+    L.or_ss_scale(raw.shape[0], _p(raw), _p(_f64(mins)), _p(_f64(maxs)), _p(out))
+    return out
+
+
+def ss_fit(raw, init_idx, pcs=8, max_iter=100):
+    """The whole oracle fit chain: preprocess -> PCA -> project -> K-Means."""
+    X, mins, maxs = ss_preprocess(raw)
+    mean, basis, ev = ss_pca(X, pcs)
+    Y = ss_project(X, mean, basis)
+    cent, assign, it = ss_kmeans(Y, init_idx, max_iter)
+    return {"mins": mins, "maxs": maxs, "mean": mean, "basis": basis, "eigval": ev, "centroids": cent,
+            "assign": assign, "iters": it}
+
+
+def ss_predict(fit, raw):
+    X = ss_scale(raw, fit["mins"], fit["maxs"])
+    return ss_assign(ss_project(X, fit["mean"], fit["basis"]), fit["centroids"])

@@ -270,3 +270,14 @@ double or_ss_vote_expected_accuracy(const int64_t *counts, int nfmt, int draws, 
   free(h);
   return acc;
 }
+
+/* Scale new matrices with the fitted ranges (prediction path): transform, then
+   (v - lo) / (hi - lo) per column (0 for a constant training column). */
+void or_ss_scale(int64_t n, const double *raw, const double *mins, const double *maxs, double *out) {
+  for (int64_t i = 0; i < n; i++)
+    for (int j = 0; j < OR_NFEAT; j++) {
+      double v = raw[i * OR_NFEAT + j];
+      double t = kind_of[j] == 0 ? log1p(v) : sqrt(v);
+      out[i * OR_NFEAT + j] = maxs[j] > mins[j] ? (t - mins[j]) / (maxs[j] - mins[j]) : 0.0;
+    }
+}

@@ -302,3 +302,104 @@ class _DevView:
     def __init__(self, ptr: int, n: int, typestr: str):
         self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3,
                                          "strides": None}
+
+
+# ------------------------------------------------------------------ semi-supervised predictor (f1)
+NFEAT = 21
+
+
+class ClusterOpts(ctypes.Structure):
+    _fields_ = [("nc", _I32), ("pcs", _I32), ("max_iter", _I32)]
+
+
+class ClusterInfo(ctypes.Structure):
+    _fields_ = [("n", _I64), ("nc", _I32), ("pcs", _I32), ("iters", _I32), ("assign", _P), ("centroids", _P),
+                ("basis", _P), ("eigval", _P), ("mins", _P), ("maxs", _P), ("mean", _P)]
+
+
+_cl_ready = False
+
+
+def _cl():
+    global _cl_ready
+    L = lib()
+    if not _cl_ready:
+        L.sfs_features_table1.argtypes = [ctypes.POINTER(FeaturesStruct), _I64, _P]
+        L.sfs_cluster_fit.argtypes = [_P, _I64, _P, ctypes.POINTER(ClusterOpts), ctypes.POINTER(_P), _P]
+        L.sfs_cluster_vote.argtypes = [_P, _P, _P, _P]
+        L.sfs_cluster_predict.argtypes = [_P, _P, _I64, _P, _P]
+        L.sfs_cluster_describe.argtypes = [_P, ctypes.POINTER(ClusterInfo)]
+        L.sfs_cluster_free.argtypes = [_P]
+        for fn in ("sfs_features_table1", "sfs_cluster_fit", "sfs_cluster_vote", "sfs_cluster_predict",
+                   "sfs_cluster_describe", "sfs_cluster_free"):
+            getattr(L, fn).restype = _I32
+        _cl_ready = True
+    return L
+
+
+def features_table1(feats):
+    """n x 21 Table-1 matrix (P:L79–102 order) from feature dicts (sfs_features_table1)."""
+    import numpy as np
+    n = len(feats)
+    arr = (FeaturesStruct * max(n, 1))()
+    for i, f in enumerate(feats):
+        arr[i] = FeaturesStruct(*[f[k] for k in FEATURE_INT_FIELDS], *[f[k] for k in FEATURE_FLOAT_FIELDS],
+                                f["admissible_mask"], f.get("csr_variant", 0))
+    out = np.empty((n, NFEAT), np.float64)
+    _check(_cl().sfs_features_table1(arr, n, out.ctypes.data), "sfs_features_table1")
+    return out
+
+
+class ClusterModel:
+    """Fitted semi-supervised predictor (sfs_cluster_model): transform, min-max, PCA, K-Means."""
+
+    def __init__(self, table1, init_idx, nc=None, pcs=8, max_iter=100, stream=None):
+        import numpy as np
+        self._np = np
+        t = np.ascontiguousarray(table1, dtype=np.float64).reshape(-1, NFEAT)
+        init = np.ascontiguousarray(init_idx, dtype=np.int32)
+        opts = ClusterOpts(len(init) if nc is None else nc, pcs, max_iter)
+        h = ctypes.c_void_p()
+        _check(_cl().sfs_cluster_fit(t.ctypes.data, len(t), init.ctypes.data, ctypes.byref(opts), ctypes.byref(h),
+                                     _stream_ptr(stream)), "sfs_cluster_fit")
+        self.handle = h.value
+        self.info = self._describe()
+
+    def _describe(self):
+        np = self._np
+        I = ClusterInfo()
+        _check(_cl().sfs_cluster_describe(self.handle, ctypes.byref(I)), "sfs_cluster_describe")
+        arr = lambda p, n, t: np.ctypeslib.as_array(ctypes.cast(p, ctypes.POINTER(t)), shape=(n,)).copy()
+        d = ctypes.c_double
+        return {"n": I.n, "nc": I.nc, "pcs": I.pcs, "iters": I.iters,
+                "assign": arr(I.assign, I.n, ctypes.c_int32),
+                "centroids": arr(I.centroids, I.nc * I.pcs, d).reshape(I.nc, I.pcs),
+                "basis": arr(I.basis, I.pcs * NFEAT, d).reshape(I.pcs, NFEAT), "eigval": arr(I.eigval, I.pcs, d),
+                "mins": arr(I.mins, NFEAT, d), "maxs": arr(I.maxs, NFEAT, d), "mean": arr(I.mean, NFEAT, d)}
+
+    def vote(self, labels, stream=None):
+        np = self._np
+        lab = np.ascontiguousarray(labels, dtype=np.int32)
+        out = np.empty(self.info["nc"], np.int32)
+        _check(_cl().sfs_cluster_vote(self.handle, lab.ctypes.data, out.ctypes.data, _stream_ptr(stream)),
+               "sfs_cluster_vote")
+        return out
+
+    def predict(self, table1, stream=None):
+        np = self._np
+        t = np.ascontiguousarray(table1, dtype=np.float64).reshape(-1, NFEAT)
+        out = np.empty(len(t), np.int32)
+        _check(_cl().sfs_cluster_predict(self.handle, t.ctypes.data, len(t), out.ctypes.data, _stream_ptr(stream)),
+               "sfs_cluster_predict")
+        return out
+
+    def free(self):
+        if self.handle:
+            _cl().sfs_cluster_free(self.handle)
+            self.handle = None
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass

@@ -839,4 +839,61 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   return SFS_OK;
 }
 
+// ---------------------------------------------------------------- semi-supervised predictor (f1)
+sfs_status sfs_features_table1(const sfs_features_t* f, int64_t n, double* out) {
+  if (n < 0 || (n > 0 && (!f || !out))) return fail(SFS_ERR_INVALID_ARG, "null argument");
+  for (int64_t i = 0; i < n; i++) {
+    const sfs_features_t& F = f[i];
+    const double row[SFS_NFEAT] = {(double)F.nrows,     (double)F.ncols,    (double)F.nnz,        F.nnz_frac,
+                                   F.nnz_mu,            (double)F.nnz_min,  (double)F.nnz_max,    F.nnz_sig,
+                                   F.max_mu,            F.mu_min,           (double)F.csr_max,    F.sig_lower,
+                                   F.sig_higher,        (double)F.hyb_ell_size, (double)F.hyb_coo, F.hyb_ell_frac,
+                                   (double)F.diagonals, (double)F.dia_size, F.dia_frac,           F.ell_frac,
+                                   (double)F.ell_size};
+    memcpy(out + i * SFS_NFEAT, row, sizeof(row));
+  }
+  return SFS_OK;
+}
+
+sfs_status sfs_cluster_fit(const double* table1, int64_t n, const int32_t* init_idx, const sfs_cluster_opts* opt,
+                           sfs_cluster_model* out, void* stream) {
+  if (!table1 || !init_idx || !opt || !out || n < 1) return fail(SFS_ERR_INVALID_ARG, "null argument / empty corpus");
+  if (opt->nc < 1 || opt->nc > n || opt->pcs < 1 || opt->pcs > 16 || opt->max_iter < 1)
+    return fail(SFS_ERR_INVALID_ARG, "need 1 <= nc <= n, 1 <= pcs <= 16, max_iter >= 1");
+  if ((size_t)opt->nc * opt->pcs * sizeof(double) > 200 * 1024) return fail(SFS_ERR_UNSUPPORTED, "nc * pcs too large");
+  for (int c = 0; c < opt->nc; c++)
+    if (init_idx[c] < 0 || init_idx[c] >= n) return fail(SFS_ERR_INVALID_ARG, "init index out of range");
+  ClusterModel* M = cluster_new();
+  cudaError_t e = cluster_fit(table1, n, init_idx, opt->nc, opt->pcs, opt->max_iter, M, (cudaStream_t)stream);
+  if (e != cudaSuccess) {
+    cluster_free(M);
+    return cuda_fail(e, "cluster fit");
+  }
+  *out = (sfs_cluster_model)M;
+  return SFS_OK;
+}
+
+sfs_status sfs_cluster_vote(sfs_cluster_model Mh, const int32_t* labels, int32_t* cluster_label, void* stream) {
+  if (!Mh || !labels || !cluster_label) return fail(SFS_ERR_INVALID_ARG, "null argument");
+  cudaError_t e = cluster_vote((const ClusterModel*)Mh, labels, cluster_label, (cudaStream_t)stream);
+  return e == cudaSuccess ? SFS_OK : cuda_fail(e, "cluster vote");
+}
+
+sfs_status sfs_cluster_predict(sfs_cluster_model Mh, const double* table1, int64_t q, int32_t* cluster, void* stream) {
+  if (!Mh || !table1 || !cluster || q < 1) return fail(SFS_ERR_INVALID_ARG, "null argument");
+  cudaError_t e = cluster_predict((const ClusterModel*)Mh, table1, q, cluster, (cudaStream_t)stream);
+  return e == cudaSuccess ? SFS_OK : cuda_fail(e, "cluster predict");
+}
+
+sfs_status sfs_cluster_describe(sfs_cluster_model Mh, sfs_cluster_info* out) {
+  if (!Mh || !out) return fail(SFS_ERR_INVALID_ARG, "null argument");
+  cluster_info((const ClusterModel*)Mh, out);
+  return SFS_OK;
+}
+
+sfs_status sfs_cluster_free(sfs_cluster_model Mh) {
+  cluster_free((ClusterModel*)Mh);
+  return SFS_OK;
+}
+
 }  // extern "C"

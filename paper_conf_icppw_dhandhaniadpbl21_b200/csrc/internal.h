@@ -101,6 +101,16 @@ int csr_vector_tpv(long long m, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
 cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s);
 
+// ---------------------------------------------------------------- semi-supervised predictor (cluster.cu)
+struct ClusterModel;
+cudaError_t cluster_fit(const double* raw, long long n, const int* init_idx, int nc, int k, int max_iter,
+                        ClusterModel* M, cudaStream_t s);
+cudaError_t cluster_vote(const ClusterModel* M, const int* labels, int* out, cudaStream_t s);
+cudaError_t cluster_predict(const ClusterModel* M, const double* raw, long long q, int* cluster, cudaStream_t s);
+ClusterModel* cluster_new();
+void cluster_free(ClusterModel* M);
+void cluster_info(const ClusterModel* M, sfs_cluster_info* out);
+
 // ---------------------------------------------------------------- matrix handle
 struct Matrix {
   int fmt = 0, dtype = 0;
