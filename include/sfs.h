@@ -76,7 +76,8 @@ typedef struct {
       ell_frac;
   uint32_t admissible_mask; /* bit f set iff format f is admissible (Q11) */
   int32_t csr_variant;      /* CSR kernel the library picks for this matrix (Q17): 0 vector (CUSP
-                               mapping), 1 merge path, 2 stream (warp per 32 rows) */
+                               mapping), 1 merge path, 2 stream (warp per 32 rows), 3 tile
+                               (nnz-balanced 256-entry chunks, rows rebuilt from row_ptr) */
 } sfs_features_t;
 
 typedef struct sfs_matrix_ *sfs_matrix; /* opaque, library-owned */
@@ -107,7 +108,7 @@ typedef struct {
   int64_t fill_slack;    /* (1<<20) */
   double hyb_rel_speed;  /* Q6 HYB width rule (3.0) */
   int64_t hyb_breakeven; /* (4096) */
-  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream */
+  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream; 3 = tile */
   int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (0: direct launches with PDL) */
 } sfs_race_opts;
 

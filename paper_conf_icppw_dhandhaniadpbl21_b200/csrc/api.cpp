@@ -178,10 +178,15 @@ static void finalize(long long m, long long n, long long z, const DevAggr& a, lo
   if (f->ell_size <= lim) mask |= 1u << SFS_ELL;
   if (f->dia_size <= lim) mask |= 1u << SFS_DIA;
   f->admissible_mask = mask;
-  // Q17: CSR stream kernel (warp per 32 rows) unless row lengths are skewed, then merge path
+  // Q17 (measured on corpus-200): merge path when empty rows are common (more than one
+  // per 256-entry chunk on average: a tile chunk would zero long runs of them, merge tiles count rows
+  // as work); else the tile kernel (nnz-balanced chunks) for skewed rows or nnz >= 2^20; else the
+  // stream kernel (warp per 32 rows), whose single launch is fastest on small regular matrices.
   const long long avg = std::max(1LL, z / m);
-  f->csr_variant = (mx <= 4 * avg + 32) ? 2 : 1;
-  if (o.csr_variant >= 0 && o.csr_variant <= 2) f->csr_variant = o.csr_variant;
+  if (a.empty_rows * 256 > (long long)z) f->csr_variant = 1;
+  else if (mx > 4 * avg + 32 || z >= (1LL << 20)) f->csr_variant = 3;
+  else f->csr_variant = 2;
+  if (o.csr_variant >= 0 && o.csr_variant <= 3) f->csr_variant = o.csr_variant;
 }
 
 static sfs_status check_csr(const sfs_csr* A) {
@@ -358,6 +363,10 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         A->work = own(csr_merge_work_bytes(m, z, d.dtype));
         if (!A->work) return bail(SFS_ERR_OOM, "csr merge carries");
         TRY_CUDA(launch_csr_merge_prepare((const int*)A->ptr[0], m, z, A->work, s));
+      } else if (A->variant == 3 && z > 0) {
+        A->work = own(csr_tile_work_bytes(m, z));
+        if (!A->work) return bail(SFS_ERR_OOM, "csr tile partition");
+        TRY_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, s));
       }
       break;
     }

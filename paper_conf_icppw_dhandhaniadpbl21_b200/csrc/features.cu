@@ -174,6 +174,7 @@ __global__ void k_popcount(const unsigned* __restrict__ bitmap, long long words,
 // bins [kHistCap - 128(l+1), kHistCap - 128 l), i.e. lane 0 the longest lengths.
 __global__ void k_hyb_select(long long m, long long j, DevAggr* __restrict__ ag, const unsigned* __restrict__ hist) {
   const int l = threadIdx.x;
+  if (l == 0) ag->empty_rows = hist[0];
   const long long mx = (long long)ag->max_len;
   const long long bc = (long long)ag->big_cnt, bs = (long long)ag->big_sum;
   if (mx == 0) {

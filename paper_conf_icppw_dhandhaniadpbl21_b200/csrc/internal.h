@@ -44,7 +44,8 @@ struct DevAggr {                // zeroed by memset; every field updated with at
   unsigned long long big_cnt, big_sum;  // rows with len >= kHistCap
   long long hyb_k;                      // -1: order statistic beyond the histogram, host refines
   long long hyb_coo;
-  long long pad[2];
+  long long empty_rows;                 // rows of length 0 (hist[0]; csr variant choice, Q17)
+  long long pad[1];
 };
 
 enum : unsigned long long {
@@ -97,6 +98,8 @@ int spmv_kernels_per_call(const Matrix* A);
 cudaError_t launch_spmv(const Matrix* A, const void* x, void* y, cudaStream_t s);
 size_t csr_merge_work_bytes(long long m, long long z, int dtype);
 cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s);
+size_t csr_tile_work_bytes(long long m, long long z);
+cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s);
 int csr_vector_tpv(long long m, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
 cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s);
@@ -119,8 +122,8 @@ struct Matrix {
   void* owned[8] = {nullptr};  // buffers to free
   int n_owned = 0;
   long long bytes = 0;
-  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream
-  void* work = nullptr;        // CSR merge carries
+  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile
+  void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;
 };
 

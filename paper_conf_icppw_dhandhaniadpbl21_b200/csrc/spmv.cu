@@ -402,6 +402,195 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
   pdl_trigger();
 }
 
+// ======================================================================== CSR tile (nnz-balanced)
+// The COO kernel's shape on the CSR arrays.  Warp w streams the contiguous chunks [cb, ce) of 256
+// entries (8 per lane, 256-bit col/val loads whose addresses do not depend on row_ptr), and the row of
+// every entry is rebuilt in shared memory from the chunk's slice of row_ptr, off the col -> x chain:
+// the rows that START in chunk c are [a_c, a_{c+1}), a_c = lower_bound(rp[0..m), 256 c) (computed
+// once per matrix); each non-empty one marks its start position, a max-scan carries the marks to
+// every entry, seeded with a_c - 1 (the row open at the chunk start).  Empty rows are zeroed by the
+// chunk that owns them.  Rows starting inside the warp's range are finished with plain stores; the
+// one row open at the range start goes to a per-warp carry that the fixup kernel adds (atomically,
+// after this grid completes).  No zero pass, no row array: CSR's own bytes only.
+constexpr int kTThreads = 256;
+constexpr int kTV = 8;
+constexpr int kTChunk = 32 * kTV;
+
+struct TileGeom {
+  long long nchunks, cpw, nwarps;
+};
+TileGeom tile_geom(long long z) {
+  TileGeom g;
+  g.nchunks = ceil_div(z, kTChunk);
+  const long long max_warps = (long long)kSMs * 4 * (kTThreads / 32);  // one resident wave at 4 CTAs / SM
+  g.cpw = ceil_div(g.nchunks, max_warps) < 1 ? 1 : ceil_div(g.nchunks, max_warps);
+  g.nwarps = ceil_div(g.nchunks, g.cpw);
+  return g;
+}
+
+__global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, long long nchunks, int* __restrict__ a) {
+  for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c <= nchunks;
+       c += (long long)gridDim.x * blockDim.x) {
+    long long v;
+    if (c == 0) v = 0;
+    else if (c == nchunks) v = m;
+    else {
+      const long long k = c * kTChunk;
+      long long lo = 0, hi = m;  // first row r with rp[r] >= k
+      while (lo < hi) {
+        const long long mid = (lo + hi) >> 1;
+        if (rp[mid] < k) lo = mid + 1;
+        else hi = mid;
+      }
+      v = lo;
+    }
+    a[c] = (int)v;
+  }
+}
+
+template <typename T, bool VEC>
+__device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const int* __restrict__ col,
+                                              const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
+                                              long long m, long long z, long long cpw, long long warp,
+                                              const int* __restrict__ ca, int* __restrict__ carry_row,
+                                              acc_t* __restrict__ carry_val, int* head) {
+  const int l = threadIdx.x & 31;
+  const long long nchunks = ceil_div(z, kTChunk);
+  const long long cb = warp * cpw;
+  const long long ce = cb + cpw < nchunks ? cb + cpw : nchunks;
+  const int own_lo = __ldg(ca + cb);  // rows >= own_lo start inside this range
+  int open_row = -1;                  // row left open at the previous chunk's end (all lanes agree)
+  acc_t open = 0;
+  int out_row = (int)m;               // the row open at the range start, for the fixup
+  acc_t out_val = 0;
+  auto emit = [&](int row, acc_t v) {
+    if (row < own_lo) { out_row = row; out_val = v; }
+    else y[row] = (T)v;
+  };
+  for (long long ch = cb; ch < ce; ch++) {
+    const long long k0 = ch * kTChunk;
+    const long long k = k0 + l * kTV;
+    const int a_lo = __ldg(ca + ch), a_hi = __ldg(ca + ch + 1);
+    acc_t p[kTV];
+    {
+      int c[kTV];
+      T v[kTV];
+      if (VEC && k + kTV <= z) {
+        ld_stream8(col + k, c);  // 32 B aligned: k is a multiple of 8, the bases were checked on the host
+        ld_stream8(val + k, v);
+      } else {
+#pragma unroll
+        for (int i = 0; i < kTV; i++) {
+          const long long kk = k + i < z ? k + i : z - 1;  // padding: a valid column, value 0
+          c[i] = ld_stream(col + kk);
+          v[i] = k + i < z ? ld_stream(val + kk) : T(0);
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < kTV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
+    }
+    // start marks of the rows beginning in this chunk (non-empty rows start at distinct positions)
+    reinterpret_cast<int4*>(head)[2 * l] = make_int4(-1, -1, -1, -1);
+    reinterpret_cast<int4*>(head)[2 * l + 1] = make_int4(-1, -1, -1, -1);
+    __syncwarp();
+    for (int r = a_lo + l; r < a_hi; r += 32) {
+      const int b = __ldg(rp + r), e = __ldg(rp + r + 1);
+      if (e > b) head[b - k0] = r;
+      else y[r] = T(0);
+    }
+    __syncwarp();
+    int r[kTV];
+    {
+      const int4 h0 = reinterpret_cast<const int4*>(head)[2 * l], h1 = reinterpret_cast<const int4*>(head)[2 * l + 1];
+      const int hv[kTV] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
+      int run = -1;
+#pragma unroll
+      for (int i = 0; i < kTV; i++) {
+        run = hv[i] > run ? hv[i] : run;
+        r[i] = run;
+      }
+      int inc = run;  // warp inclusive max-scan of the lane maxima
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (l >= o) inc = u > inc ? u : inc;
+      }
+      int ex = __shfl_up_sync(0xffffffffu, inc, 1);
+      if (l == 0 || ex < a_lo - 1) ex = a_lo - 1;
+#pragma unroll
+      for (int i = 0; i < kTV; i++) r[i] = r[i] > ex ? r[i] : ex;
+    }
+    __syncwarp();  // head is rewritten by the next chunk
+    // segmented reduction of (r[i], p[i]) exactly as in the COO kernel; padding items (past z) have
+    // p = 0 and the last row
+    const int rf = r[0], rl = r[kTV - 1];
+    const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
+    if (open_row >= 0 && open_row != chunk_first) {
+      if (l == 0) emit(open_row, open);
+      open_row = -1;
+      open = 0;
+    }
+    acc_t hsum = p[0], cur = p[0];
+    int cr = rf;
+    bool in_head = true;
+#pragma unroll
+    for (int i = 1; i < kTV; i++) {
+      if (r[i] != cr) {
+        if (in_head) { hsum = cur; in_head = false; }
+        else emit(cr, cur);
+        cr = r[i];
+        cur = p[i];
+      } else {
+        cur += p[i];
+      }
+    }
+    if (in_head) hsum = cur;
+    const bool single = (rf == rl);
+    const acc_t in0 = (open_row == rf) ? open : acc_t(0);
+    const int prev_rl = __shfl_up_sync(0xffffffffu, rl, 1);
+    int f = (l == 0) || !single || (prev_rl != rf);
+    acc_t S = cur + ((l == 0 && single) ? in0 : acc_t(0));
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const acc_t us = __shfl_up_sync(0xffffffffu, S, o);
+      const int uf = __shfl_up_sync(0xffffffffu, f, o);
+      if (l >= o) {
+        if (!f) S += us;
+        f |= uf;
+      }
+    }
+    const acc_t S_prev = __shfl_up_sync(0xffffffffu, S, 1);
+    const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
+    if (!single) emit(rf, hsum + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0))));
+    if (l < 31 && next_rf != rl) emit(rl, S);
+    open_row = __shfl_sync(0xffffffffu, rl, 31);
+    open = __shfl_sync(0xffffffffu, S, 31);
+  }
+  if (l == 0 && open_row >= 0) emit(open_row, open);  // a partial if the row continues past the range
+  const unsigned has = __ballot_sync(0xffffffffu, out_row < m);
+  if (has) {
+    if (l == __ffs(has) - 1) { carry_row[warp] = out_row; carry_val[warp] = out_val; }
+  } else if (l == 0) {
+    carry_row[warp] = (int)m;
+  }
+}
+
+// blockDim is 64, 128 or 256 (smaller CTAs spread a small matrix's few warps over more SMs)
+template <typename T, bool VEC>
+__global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
+                                                               const T* __restrict__ val, const T* __restrict__ x,
+                                                               T* __restrict__ y, long long m, long long z,
+                                                               long long cpw, long long nwarps,
+                                                               const int* __restrict__ ca, int* __restrict__ carry_row,
+                                                               acc_t* __restrict__ carry_val) {
+  __shared__ __align__(16) int s_head[kTThreads / 32][kTChunk];
+  pdl_wait();
+  pdl_trigger();  // the fixup kernel launches now and waits for this grid to finish
+  const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (warp < nwarps)
+    csr_tile_warp<T, VEC>(rp, col, val, x, y, m, z, cpw, warp, ca, carry_row, carry_val, s_head[threadIdx.x >> 5]);
+}
+
 // ======================================================================== COO (also the COO part of HYB)
 constexpr int kCooThreads = 256;
 constexpr int kCooV = 8;                // items per lane per step (two 128-bit loads per array)
@@ -714,6 +903,22 @@ MergeWork merge_work(void* base, long long tiles) {
   return w;
 }
 
+struct TileWork {
+  int* a;
+  int* crow;
+  acc_t* cval;
+};
+TileWork tile_work(void* base, const TileGeom& g) {
+  TileWork w;
+  char* p = (char*)base;
+  w.a = (int*)p;
+  p += al256(sizeof(int) * (g.nchunks + 1));
+  w.crow = (int*)p;
+  p += al256(sizeof(int) * g.nwarps);
+  w.cval = (acc_t*)p;
+  return w;
+}
+
 // COO launch geometry: contiguous chunk ranges, one resident wave of warps at most.
 template <typename T, bool ACCUM>
 cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
@@ -749,7 +954,28 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       const int* rp = (const int*)A->ptr[0];
       const int* col = (const int*)A->ptr[1];
       const T* val = (const T*)A->ptr[2];
-      if (A->variant == 2) {
+      if (A->variant == 3) {
+        if (z == 0) {
+          e = launch_zero<T>(y, m, s);
+          break;
+        }
+        const TileGeom g = tile_geom(z);
+        TileWork w = tile_work(A->work, g);
+        // small matrices: fewer warps per CTA so that the CTAs cover >= 2 x 148 SMs where possible
+        int tpb = kTThreads;
+        while (tpb > 64 && ceil_div(g.nwarps, tpb / 32) < 2 * kSMs) tpb >>= 1;
+        const dim3 grid((unsigned)ceil_div(g.nwarps, tpb / 32));
+        // borrowed arrays (e.g. a row block of a larger CSR) may not be 32 B aligned: scalar loads
+        const bool vec = ((((uintptr_t)col) | ((uintptr_t)val)) % 32) == 0;
+        auto go = [&](auto kern) {
+          return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a, w.crow,
+                          w.cval);
+        };
+        e = vec ? go(k_spmv_csr_tile<T, true>) : go(k_spmv_csr_tile<T, false>);
+        if (e == cudaSuccess)
+          e = launch_k(k_spmv_csr_merge_fixup<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, (const int*)w.crow,
+                       (const acc_t*)w.cval, g.nwarps, m, y);
+      } else if (A->variant == 2) {
         const long long groups = ceil_div(m, 32);
         const long long windows = ceil_div(z, 32 * stream_u<T>());  // ~ windows over all groups
         const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
@@ -855,9 +1081,23 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
   return cudaGetLastError();
 }
 
+size_t csr_tile_work_bytes(long long m, long long z) {
+  (void)m;
+  const TileGeom g = tile_geom(z);
+  return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) + al256(sizeof(acc_t) * g.nwarps);
+}
+
+cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s) {
+  const TileGeom g = tile_geom(z);
+  TileWork w = tile_work(work, g);
+  k_csr_tile_partition<<<grid_cap(g.nchunks + 1, 256, 8), 256, 0, s>>>(rp, m, g.nchunks, w.a);
+  count_launch();
+  return cudaGetLastError();
+}
+
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
-    case SFS_CSR: return A->variant == 1 ? 2 : 1;
+    case SFS_CSR: return (A->variant == 1 || (A->variant == 3 && A->nnz > 0)) ? 2 : 1;
     case SFS_COO: return A->nnz > 0 ? 2 : 1;
     case SFS_HYB: return A->coo_nnz > 0 ? 2 : 1;
     default: return 1;

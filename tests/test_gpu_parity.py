@@ -75,7 +75,7 @@ def test_conversions_bit_exact(name):
 
 
 @pytest.mark.parametrize("name", NAMES)
-@pytest.mark.parametrize("variant", [0, 1, 2])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3])
 def test_spmv_tolerance(name, variant):
     A = cases()[name]
     fo = oracle.features(A.m, A.n, A.rp, A.col)
@@ -103,7 +103,7 @@ def test_spmv_x_ones_bitwise(dtype, cls, N, pts):
     dA = to_dev(A)
     tdt = torch.float64 if dtype == sfsgen.F64 else torch.float32
     x = torch.ones(A.n, dtype=tdt, device="cuda")
-    for variant in (0, 1, 2):
+    for variant in (0, 1, 2, 3):
         for fmt in range(5):
             if variant != 2 and fmt != sfs.CSR:
                 continue
@@ -231,3 +231,59 @@ def test_launch_count_increases():
     for _ in range(3):
         sfs.spmv(sfs.COO, M, x, y)
     assert sfs.launch_count() - c0 == 6  # memset + kernel per COO SpMV
+
+
+def _tile_edge_csr(dtype, cap=None):
+    """Rows that stress the CSR tile kernel (variant 3): leading / trailing / mid-matrix runs of empty
+    rows, rows of exactly 255/256/257/512 entries, one row of 400,000 entries spanning many warp
+    ranges, and nnz large enough (> 148*4*8 chunks of 256) that each warp owns several chunks.
+    cap: clip row lengths (cap = 256 selects the carry-free mode, every row <= one chunk)."""
+    rng = np.random.default_rng(77)
+    m, n = 200_000, 500_000
+    lens = rng.poisson(6, m).astype(np.int64)
+    lens[:1000] = 0
+    lens[-5000:] = 0
+    lens[90_000:93_000] = 0
+    lens[rng.integers(0, m, 20_000)] = 0
+    lens[[5000, 5001, 5002, 77_777]] = [255, 256, 257, 512]
+    lens[123_456] = 400_000
+    if cap is not None:
+        lens = np.minimum(lens, cap)
+        lens[rng.integers(0, m, 3000)] = cap  # many rows of exactly one chunk
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    z = int(rp[-1])
+    col = np.empty(z, np.int64)
+    starts = rng.integers(0, n - 3 * 1000, m)
+    for r in np.nonzero(lens)[0]:
+        L = int(lens[r])
+        if L >= 1000:
+            col[rp[r]:rp[r + 1]] = np.sort(rng.choice(n, L, replace=False))
+        else:
+            col[rp[r]:rp[r + 1]] = starts[r] + np.cumsum(rng.integers(1, 4, L))
+    val = rng.uniform(0.5, 1.0, z) * rng.choice([-1.0, 1.0], z)
+    return sfsgen.CSR(m, n, rp.astype(np.int32), col.astype(np.int32),
+                      val.astype(np.float64 if dtype == sfsgen.F64 else np.float32))
+
+
+@pytest.mark.parametrize("cap", [None, 256])
+@pytest.mark.parametrize("dtype", [sfsgen.F64, sfsgen.F32])
+def test_csr_tile_edges(dtype, cap):
+    import torch
+    A = _tile_edge_csr(dtype, cap)
+    x = sfsgen.vector(5, A.n, A.dtype)
+    dA = to_dev(A)
+    M = sfs.convert(dA, sfs.CSR, sfs.default_opts(csr_variant=3))
+    assert M.layout().variant == 3
+    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="tile-edges")
+    M.free()
+    # borrowed arrays that are not 32 B aligned (a view at an element offset): scalar-load path
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    colb = torch.empty(A.nnz + 1, dtype=torch.int32, device="cuda")
+    valb = torch.empty(A.nnz + 1, dtype=t(A.val).dtype, device="cuda")
+    colb[1:] = t(A.col)
+    valb[1:] = t(A.val)
+    dB = sfs.Csr(A.m, A.n, t(A.rp), colb[1:], valb[1:])
+    M = sfs.convert(dB, sfs.CSR, sfs.default_opts(csr_variant=3))
+    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="tile-edges-misaligned")
+    M.free()

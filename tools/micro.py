@@ -48,7 +48,8 @@ def main():
     ap.add_argument("--formats", default="CSR,COO,ELL,HYB,DIA")
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--warmup", type=int, default=5)
-    ap.add_argument("--variant", type=int, default=-1, help="CSR kernel: -1 auto (Q17), 0 vector, 1 merge")
+    ap.add_argument("--variant", type=int, default=-1, help="CSR kernel: -1 auto (Q17), 0 vector, 1 merge, 2 stream")
+    ap.add_argument("--variants", default=None, help="comma list: time CSR once per variant (CSR/v keys)")
     ap.add_argument("--json", default=None)
     ap.add_argument("--no-cold", action="store_true")
     args = ap.parse_args()
@@ -58,7 +59,12 @@ def main():
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
     import sfsgen
 
-    A = make_matrix(args.matrix)
+    for name in args.matrix.split(","):
+        run_one(args, name, torch, sfs, sfsgen)
+
+
+def run_one(args, matrix, torch, sfs, sfsgen):
+    A = make_matrix(matrix)
     x = sfsgen.vector(3, A.n, A.dtype)
     t = lambda a: torch.from_numpy(a).cuda()
     dA = sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val))
@@ -75,10 +81,17 @@ def main():
         pass
     # feature pass time
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    out = {"matrix": args.matrix, "m": A.m, "n": A.n, "nnz": A.nnz, "dtype": "f64" if A.dtype else "f32",
+    out = {"matrix": matrix, "m": A.m, "n": A.n, "nnz": A.nnz, "dtype": "f64" if A.dtype else "f32",
            "peak_gbs": peak, "formats": {}}
+    jobs = []
     for name in args.formats.split(","):
-        fmt = sfs.FORMAT_NAMES.index(name)
+        if name == "CSR" and args.variants:
+            jobs += [(f"CSR/{v}", int(v)) for v in args.variants.split(",")]
+        else:
+            jobs.append((name, args.variant))
+    for name, variant in jobs:
+        opts = sfs.default_opts(csr_variant=variant)
+        fmt = sfs.FORMAT_NAMES.index(name.split("/")[0])
         if not (feats["admissible_mask"] >> fmt) & 1:
             out["formats"][name] = "inadmissible"
             continue
@@ -115,7 +128,8 @@ def main():
         out["formats"][name] = res
         M.free()
     s = json.dumps(out)
-    print(s)
+    print(f"{matrix:14s} m={A.m} nnz={A.nnz} " + "  ".join(
+        f"{k} {v['hot_us']:.1f}us {v['hot_gbs']:.0f}GB/s" for k, v in out["formats"].items() if isinstance(v, dict)))
     if args.json:
         with open(args.json, "a") as fh:
             fh.write(s + "\n")
