@@ -399,13 +399,16 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       void* cv = own(sv * std::max(nc, 1LL));
       if (!ec || !ev || !cr || !cc || !cv) return bail(SFS_ERR_OOM, "hyb");
       TRY_CUDA(launch_csr2ell(d.dtype, d.rp, d.col, d.val, m, P, (int)K, ec, ev, s));
+      // rows overflowing by <= kHybRowwiseMax: keep the per-row overflow offsets for the one-launch SpMV
+      A->variant = hyb_rowwise(f.nnz_max, K, nc, z);
       if (nc > 0) {
         Temps t(s);
-        int* ovf = (int*)t.get(sizeof(int) * (m + 1));
+        int* ovf = A->variant ? (int*)own(sizeof(int) * (m + 1)) : (int*)t.get(sizeof(int) * (m + 1));
         void* work = t.get(scan_work_bytes(m));
         if (!ovf || !work) return bail(SFS_ERR_OOM, "hyb scan");
         TRY_CUDA(launch_overflow_scan(d.rp, m, (int)K, ovf, work, s));
         TRY_CUDA(launch_hyb_coo_part(d.dtype, d.rp, d.col, d.val, m, z, (int)K, ovf, cr, cc, cv, s));
+        if (A->variant) A->ptr[5] = ovf;
       }
       A->ptr[0] = ec; A->ptr[1] = ev; A->ptr[2] = cr; A->ptr[3] = cc; A->ptr[4] = cv;
       A->width = K;

@@ -101,6 +101,7 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 size_t csr_tile_work_bytes(long long m, long long z);
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s);
 int csr_vector_tpv(long long m, long long z);
+int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
 cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s);
 
@@ -122,7 +123,7 @@ struct Matrix {
   void* owned[8] = {nullptr};  // buffers to free
   int n_owned = 0;
   long long bytes = 0;
-  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile
+  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile; HYB: 1 = one launch (ptr[5] = ovf)
   void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;
 };

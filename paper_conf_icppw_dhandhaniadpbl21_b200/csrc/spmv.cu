@@ -41,6 +41,13 @@ constexpr long long kResidentThreads = (long long)kSMs * 2048;
 
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+// SFS_PDL_EARLY: release the successor right after our own wait (it is scheduled once all our CTAs
+// are resident, then blocks in griddepcontrol.wait until this grid has completed and flushed).
+#ifdef SFS_PDL_EARLY
+__device__ __forceinline__ void pdl_early() { pdl_trigger(); }
+#else
+__device__ __forceinline__ void pdl_early() {}
+#endif
 
 bool pdl_enabled() {
   static int v = -1;
@@ -120,6 +127,7 @@ __global__ void __launch_bounds__(256) k_spmv_csr_vector(const int* __restrict__
                                                          const T* __restrict__ val, const T* __restrict__ x,
                                                          T* __restrict__ y, long long m) {
   pdl_wait();
+  pdl_early();
   const long long gt = (long long)blockIdx.x * blockDim.x + threadIdx.x;
   const int lane = threadIdx.x & (TPV - 1);
   const long long V = ((long long)gridDim.x * blockDim.x) / TPV;
@@ -170,6 +178,7 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
   __shared__ acc_t sbuf[kSWarps][kSW];
   __shared__ acc_t s_part[kSWarps][32];
   pdl_wait();
+  pdl_early();
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int NG = kSWarps / S;  // groups per CTA iteration
   const int p = w / NG, gl = w % NG;
@@ -315,6 +324,7 @@ __global__ void __launch_bounds__(kMT) k_spmv_csr_merge(const int* __restrict__ 
   __shared__ acc_t s_ws[33];
   __shared__ int s_wf[32];
   pdl_wait();
+  pdl_early();
   const long long total = m + z;
   const long long d0 = (long long)blockIdx.x * kMTile;
   const long long d1 = d0 + kMTile < total ? d0 + kMTile : total;
@@ -394,6 +404,7 @@ template <typename T>
 __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const acc_t* __restrict__ carry_val,
                                        long long tiles, long long m, T* __restrict__ y) {
   pdl_wait();
+  pdl_early();
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < tiles; t += (long long)gridDim.x * blockDim.x) {
     const int r = carry_row[t];
     const acc_t v = carry_val[t];
@@ -647,6 +658,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       }
       if (!waited) {
         pdl_wait();
+        pdl_early();
         waited = true;
       }
       const int rf = r[0], rl = r[kCooV - 1];
@@ -712,15 +724,24 @@ constexpr int kEllThreads = 256;
 template <typename T> constexpr int ell_batch() { return sizeof(T) == 4 ? 8 : 4; }   // bytes in flight per thread
 template <typename T> constexpr int ell_ctas() { return sizeof(T) == 4 ? 3 : 4; }    // CTAs / SM (register cap)
 
-template <typename T>
+// OVF (HYB whose rows overflow the ELL part by at most kHybRowwiseMax entries): part 0 of each row
+// group also adds its rows' COO-part entries, located by the per-row overflow offsets ovf[0..m]
+// kept from the conversion -- HYB in one launch, y written once.
+constexpr long long kHybRowwiseMax = 32;
+
+template <typename T, bool OVF>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
                                                                          const T* __restrict__ eval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
                                                                          long long m, long long P, int K, int S,
-                                                                         int early_trigger) {
+                                                                         int early_trigger,
+                                                                         const int* __restrict__ ovf,
+                                                                         const int* __restrict__ ocol,
+                                                                         const T* __restrict__ oval) {
   constexpr int kB = ell_batch<T>();
   __shared__ acc_t s_part[kEllThreads][4];
   pdl_wait();
+  pdl_early();
   if (early_trigger) pdl_trigger();  // HYB: let the COO part start its loads now
   const int G = kEllThreads / S;
   const int p = threadIdx.x / G, g = threadIdx.x % G;
@@ -733,6 +754,11 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
     const long long r = grp * 4;
     acc_t acc[4] = {0, 0, 0, 0};
     if (grp < groups) {
+      int ob[5];
+      if (OVF && p == 0) {
+#pragma unroll
+        for (int q = 0; q <= 4; q++) ob[q] = __ldg(ovf + (r + q < m ? r + q : m));
+      }
       const int* cp = ecol + r;
       const T* vp = eval + r;
       int j = j0;
@@ -760,6 +786,30 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
         if (c.y >= 0) acc[1] += (acc_t)v.v[1] * (acc_t)ld_x(x + c.y);
         if (c.z >= 0) acc[2] += (acc_t)v.v[2] * (acc_t)ld_x(x + c.z);
         if (c.w >= 0) acc[3] += (acc_t)v.v[3] * (acc_t)ld_x(x + c.w);
+      }
+      if (OVF && p == 0) {
+        // the 4 rows' overflow entries are contiguous: [ob[0], ob[4]), 4 at a time, clamped loads
+        for (int k = ob[0]; k < ob[4]; k += 4) {
+          int c[4];
+          T v[4];
+#pragma unroll
+          for (int u = 0; u < 4; u++) {
+            const int kk = k + u < ob[4] ? k + u : ob[4] - 1;
+            c[u] = ld_stream(ocol + kk);
+            v[u] = ld_stream(oval + kk);
+          }
+#pragma unroll
+          for (int u = 0; u < 4; u++) {
+            const acc_t t = (acc_t)v[u] * (acc_t)ld_x(x + c[u]);
+            const int kk = k + u;
+            if (kk < ob[4]) {
+              if (kk < ob[1]) acc[0] += t;
+              else if (kk < ob[2]) acc[1] += t;
+              else if (kk < ob[3]) acc[2] += t;
+              else acc[3] += t;
+            }
+          }
+        }
       }
     }
     if (S > 1) {
@@ -805,6 +855,7 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
   __shared__ int s_off[kDiaSmemOffs];
   __shared__ acc_t s_part[S > 1 ? kDiaThreads * kR : 1];
   pdl_wait();
+  pdl_early();
   const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
   for (int i = threadIdx.x; i < nsm; i += blockDim.x) s_off[i] = offs[i];
   __syncthreads();
@@ -941,8 +992,11 @@ cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s,
   const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
   const long long niter = ceil_div(groups, kEllThreads / S);
   const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
-  return launch_k(k_spmv_ell<T>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1], x, y,
-                  A->m, A->pitch, K, S, early_trigger);
+  if (A->fmt == SFS_HYB && A->variant == 1)
+    return launch_k(k_spmv_ell<T, true>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1],
+                    x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3], (const T*)A->ptr[4]);
+  return launch_k(k_spmv_ell<T, false>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1],
+                  x, y, A->m, A->pitch, K, S, early_trigger, (const int*)nullptr, (const int*)nullptr, (const T*)nullptr);
 }
 
 template <typename T>
@@ -1015,8 +1069,9 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
     case SFS_ELL:
     case SFS_HYB: {
       const int K = (int)A->width;
-      e = K == 0 ? launch_zero<T>(y, m, s) : launch_ell<T>(A, x, y, K, s, A->fmt == SFS_HYB && A->coo_nnz > 0);
-      if (e == cudaSuccess && A->fmt == SFS_HYB && A->coo_nnz > 0)
+      const bool two = A->fmt == SFS_HYB && A->coo_nnz > 0 && A->variant == 0;  // ELL part -> COO part
+      e = K == 0 ? launch_zero<T>(y, m, s) : launch_ell<T>(A, x, y, K, s, two);
+      if (e == cudaSuccess && two)
         e = launch_coo<T, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y, A->coo_nnz, s);
       break;
     }
@@ -1095,11 +1150,19 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
   return cudaGetLastError();
 }
 
+// One-launch HYB when the overflow per row is short: <= 4 entries at any size, <= 32 below 2^20 nnz
+// (latency-bound sizes, where the second kernel's launch edge dominates).  Measured on corpus-200:
+// longer serial overflow walks lose to the COO kernel on large random-column matrices.
+int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) {
+  const long long o = nnz_max - K;
+  return coo_nnz > 0 && (o <= 4 || (z < (1LL << 20) && o <= kHybRowwiseMax));
+}
+
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
     case SFS_CSR: return (A->variant == 1 || (A->variant == 3 && A->nnz > 0)) ? 2 : 1;
     case SFS_COO: return A->nnz > 0 ? 2 : 1;
-    case SFS_HYB: return A->coo_nnz > 0 ? 2 : 1;
+    case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? 2 : 1;
     default: return 1;
   }
 }
