@@ -277,7 +277,10 @@ def run_ours(args):
     value = total_mats / t_max
     launches_all = int(sumr(float(launches)))
 
-    # ---- e2e: same call with pinned host inputs (H2D inside the call), result D2H inside
+    # ---- e2e: same call with pinned host inputs (H2D inside the call), result D2H inside; one untimed
+    # warm-up step first (it grows the stream-ordered pool to hold the staged corpus)
+    if args.e2e_steps > 0:
+        step(hmats)
     barrier()
     e2 = torch.cuda.Event(enable_timing=True)
     e3 = torch.cuda.Event(enable_timing=True)
