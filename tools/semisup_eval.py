@@ -39,8 +39,9 @@ def mcc(y, p, K=5):
     return num / den if den else 0.0
 
 
-def macro_f1(y, p, K=5):
-    f = []
+def f1_scores(y, p, K=5):
+    """(support-weighted F1, macro F1) over the classes present in y or p (reading F4)."""
+    f, w = [], []
     for k in range(K):
         tp = np.sum((y == k) & (p == k))
         fp = np.sum((y != k) & (p == k))
@@ -48,13 +49,16 @@ def macro_f1(y, p, K=5):
         if tp + fp + fn == 0:
             continue
         f.append(2 * tp / (2 * tp + fp + fn))
-    return float(np.mean(f)) if f else 0.0
+        w.append(np.sum(y == k))
+    if not f:
+        return 0.0, 0.0
+    return float(np.dot(f, w) / max(np.sum(w), 1)), float(np.mean(f))
 
 
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("dump")
-    ap.add_argument("--nc", default="8,16,32")
+    ap.add_argument("--nc", default="8,16,32,48")
     ap.add_argument("--draws", default="1,2")
     ap.add_argument("--folds", type=int, default=5)
     ap.add_argument("--seed", type=int, default=7)
@@ -118,7 +122,8 @@ def main():
             tb, tc, tp = np.concatenate(tb), np.concatenate(tc), np.concatenate(tp)
             gt = float(np.exp(np.mean(np.log(tb / tp))))
             csr = float(np.exp(np.mean(np.log(tc / tp))))
-            res = {"nc": nc, "labels_from": mode, "ACC": float(np.mean(ys == ps)), "F1": macro_f1(ys, ps),
+            f1w, f1m = f1_scores(ys, ps)
+            res = {"nc": nc, "labels_from": mode, "ACC": float(np.mean(ys == ps)), "F1": f1w, "F1_macro": f1m,
                    "MCC": mcc(ys, ps), "GT": gt, "CSR": csr, "Threshold": int(np.sum(tp >= 1.5 * tc)),
                    "purity": float(np.mean(pur)), "fit_ms": float(np.median(fit_ms)),
                    "race_time_saved": float(np.mean(saved)) if saved else 0.0,
