@@ -1,4 +1,4 @@
-"""GPU parity at BASELINE.json's full sizes (configs[0], [2], [3] and a slice of configs[1]),
+"""GPU parity at BASELINE.json's full sizes (configs[0], [2], [3], a slice of configs[1], every generator class of configs[4] and its largest early matrix),
 through the same C-ABI calls the bench times."""
 import numpy as np
 import pytest
@@ -50,3 +50,18 @@ def test_config3_stencil3d27_128_fp64():
 def test_config1_corpus_slice(i):
     A = sfsgen.generate(sfsgen.corpus_spec(200, i))
     _full_check(A, conv=(A.nnz < 20_000_000), ctx=f"corpus200[{i}]")
+
+
+# configs[4] (SuiteSparse-shaped corpus-2000): one small matrix of every generator class (band,
+# uniform, block-diagonal, power-law, R-MAT, 2D5 / 3D7 / 3D27 stencils) fully, plus the largest of
+# the first 200 corpus-2000 matrices (features bit-exact, SpMV per row) at full size.
+@pytest.mark.parametrize("i", [1, 2, 5, 8, 12, 20, 24, 61, 75])
+def test_config4_corpus2000_classes(i):
+    A = sfsgen.generate(sfsgen.corpus_spec(2000, i))
+    _full_check(A, ctx=f"corpus2000[{i}]")
+
+
+def test_config4_corpus2000_largest_sample():
+    A = sfsgen.generate(sfsgen.corpus_spec(2000, 164))  # 47.0 M nnz, uniform random, fp64
+    assert A.nnz > 40_000_000
+    _full_check(A, conv=False, ctx="corpus2000[164]")
