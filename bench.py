@@ -60,9 +60,11 @@ def dist_env():
     return rank, world, local
 
 
-def corpus_ids(rank, per_rank):
-    """Weak scaling: rank r labels matrices [r*per_rank, (r+1)*per_rank) of the configs[1] recipe."""
-    return list(range(rank * per_rank, (rank + 1) * per_rank))
+def corpus_ids(rank, per_rank, world=1):
+    """Weak scaling: the job is the first per_rank*world matrices of the configs[1] recipe, LPT-balanced
+    over the ranks on an estimated race cost (dist.weak_shard); N = 1 labels ids [0, per_rank)."""
+    from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
+    return sd.weak_shard(200, per_rank, rank, world)
 
 
 def generate_host(ids):
@@ -217,7 +219,7 @@ def run_ours(args):
     dev = torch.device("cuda", local)
     stream = torch.cuda.current_stream()
 
-    host = generate_host(corpus_ids(rank, args.corpus))
+    host = generate_host(corpus_ids(rank, args.corpus, world))
     t = lambda a: torch.from_numpy(a).to(dev)
     mats = [sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), t(x)) for _, A, x in host]
     pin = lambda a: torch.from_numpy(a).pin_memory()
@@ -225,14 +227,20 @@ def run_ours(args):
     torch.cuda.synchronize()
     opts = sfs.default_opts(reps=args.reps, warmup=args.race_warmup, use_graphs=1 if args.graphs else 0)
     n = len(mats)
-    gather_buf = torch.zeros(n * 8, dtype=torch.float64, device=dev)
-    all_buf = torch.zeros(world * n * 8, dtype=torch.float64, device=dev)
+    n_max = n
+    if world > 1:  # LPT shards differ by a matrix or two: pad the gathered result rows
+        nt = torch.tensor([n], dtype=torch.int64, device=dev)
+        dist.all_reduce(nt, op=dist.ReduceOp.MAX)
+        n_max = int(nt.item())
+    gather_buf = torch.full((n_max * 9,), -1.0, dtype=torch.float64, device=dev)
+    all_buf = torch.zeros(world * n_max * 9, dtype=torch.float64, device=dev)
 
     def step(batch):
         feats, labs = sfs.label_corpus(batch, opts)
         if world > 1:  # a15: gather labels + timing summary to every rank (results, ~64 B / matrix)
-            rows = [[L["label"]] + L["t_spmv_us"] + [L["t_features_us"], L["matrix_status"]] for L in labs]
-            gather_buf.copy_(torch.tensor(rows, dtype=torch.float64).reshape(-1))
+            rows = [[i, L["label"]] + L["t_spmv_us"] + [L["t_features_us"], L["matrix_status"]]
+                    for (i, _, _), L in zip(host, labs)]
+            gather_buf[:n * 9].copy_(torch.tensor(rows, dtype=torch.float64).reshape(-1))
             dist.all_gather_into_tensor(all_buf, gather_buf)
         return feats, labs
 
@@ -273,7 +281,8 @@ def run_ours(args):
     launches = sfs.launch_count() - l0
     t_dev = e0.elapsed_time(e1) / 1000.0
     t_max = maxr(t_dev)
-    total_mats = world * n * args.steps
+    n_all = int(sumr(float(n)))
+    total_mats = n_all * args.steps
     value = total_mats / t_max
     launches_all = int(sumr(float(launches)))
 
@@ -293,7 +302,7 @@ def run_ours(args):
     h2d = sum(m.nbytes() + m.x.numel() * m.x.element_size() for m in hmats)
     e2e = None
     if args.e2e_steps > 0:
-        e2e = {"value": world * n * args.e2e_steps / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d,
+        e2e = {"value": n_all * args.e2e_steps / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d,
                "d2h_bytes_per_step": n * DAGGR_BYTES}
 
     # ---- roofline of the dominant kernel (from the race's own CUDA events, inside the timed region)
@@ -375,9 +384,11 @@ def run_ours(args):
                 "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": "corpus-200 (BASELINE configs[1]): banded/uniform/block-diagonal/power-law, "
                                        "10K-1M rows, values fp32 and fp64 (half each), SpMV accumulates in fp64",
-                           "matrices_per_rank": n, "nnz_per_rank": int(sum(m.nnz for m in mats)),
+                           "matrices_per_rank": n, "matrices_all_ranks": n_all,
+                           "nnz_per_rank": int(sum(m.nnz for m in mats)),
                            "reps": args.reps, "race_warmup": args.race_warmup,
-                           "parallelism": f"corpus sharded over {world} GPU(s), no data-path collective",
+                           "parallelism": f"corpus of {n_all} matrices LPT-sharded over {world} GPU(s) on estimated race "
+                                          f"cost (weak: {args.corpus} per GPU), no data-path collective",
                            "l2": "inputs larger than L2 (corpus >> 126 MB per step); in-race reps back-to-back (P:L217)"},
                 "e2e": e2e, "gpu_launches": launches_all, "clocks": clk, "roofline": roofline,
                 "cpu_baseline": cpu, "per_format": per_fmt,

@@ -38,6 +38,55 @@ def lpt_assign(costs: Sequence[float], world: int) -> List[List[int]]:
     return [sorted(s) for s in shards]
 
 
+def expected_nnz(spec) -> float:
+    """Expected nnz of a generator spec (sfsgen classes), from its parameters alone, so that every rank
+    can schedule the corpus without generating it.  Scheduling only: nothing here feeds a result.
+    band: 1 + 2b·p per row; block-diagonal: 1 + (B−1)·p; uniform: λ (dedup is negligible for n ≫ λ);
+    power-law: E[len] = 1 + Σ_{L=2}^{cap} (2/L)^(α−1) (P(len ≥ L) for the inverse-CDF draw, cap =
+    min(n, 2^17)); stencils / R-MAT: points per row / edge factor 16."""
+    import sfsgen
+    m, n = sfsgen.dims(spec)
+    c = spec.cls
+    if c == sfsgen.BAND:
+        per = 1.0 + 2.0 * spec.ia * spec.pa
+    elif c == sfsgen.BLOCKDIAG:
+        per = 1.0 + (spec.ia - 1) * spec.pa
+    elif c == sfsgen.UNIFORM:
+        per = spec.pa
+    elif c == sfsgen.POWERLAW:
+        cap = max(2, min(n, 1 << 17))
+        L = np.arange(2, cap + 1, dtype=np.float64)
+        per = 1.0 + float(np.sum((2.0 / L) ** (spec.pa - 1.0)))
+    elif c == sfsgen.RMAT:
+        per = 16.0
+    else:
+        per = {sfsgen.ST2D5: 5.0, sfsgen.ST3D7: 7.0, sfsgen.ST3D27: 27.0}.get(c, 1.0)
+    return float(m) * per
+
+
+# Race cost model of one matrix (µs): a fixed part (5 formats × 105 dependent launches at the ~3.3 µs
+# launch floor, conversions, features) plus a bandwidth part per byte of CSR (all five formats' reps),
+# least-squares fit to the corpus-200 race on a B200 (profiles/r01/corpus200_dump.jsonl, r = 0.97).
+RACE_FIXED_US = 1740.0
+RACE_US_PER_CSR_BYTE = 1.62e-4
+
+
+def race_cost(spec) -> float:
+    return RACE_FIXED_US + RACE_US_PER_CSR_BYTE * (4 + (8 if spec.dtype else 4)) * expected_nnz(spec)
+
+
+def weak_shard(corpus: int, per_rank: int, rank: int, world: int) -> List[int]:
+    """Weak scaling with balanced ranks: the job is the first per_rank·world matrices of the corpus
+    recipe, LPT-assigned over the ranks on race_cost, so every rank gets ~per_rank matrices of ~equal
+    estimated race time (world = 1: ids [0, per_rank) in order).  Identical on every rank."""
+    import sfsgen
+    ids = list(range(per_rank * world))
+    if world == 1:
+        return ids
+    costs = [race_cost(sfsgen.corpus_spec(corpus, i)) for i in ids]
+    return lpt_assign(costs, world)[rank]
+
+
 # fixed-size result row gathered across ranks: id, label, matrix status, admissible mask, csr variant,
 # t_spmv[5], t_convert[5], status[5], t_features, 23 features  -> 44 float64
 RESULT_FIELDS = 44

@@ -130,3 +130,26 @@ def test_gloo_world2_corpus_and_rowpartition():
         x, _ = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
     y = np.concatenate([y0, y1])
     assert np.allclose(y, x, rtol=1e-12, atol=0)
+
+
+def test_weak_shard_balanced():
+    """bench.py's weak scaling: the first 200·N corpus matrices, each exactly once over the ranks, with
+    estimated race costs within 2 % of each other (LPT), and N = 1 the configs[1] ids in order."""
+    import sfsgen
+    assert sd.weak_shard(200, 200, 0, 1) == list(range(200))
+    w = 4
+    sh = [sd.weak_shard(200, 50, r, w) for r in range(w)]
+    assert sorted(sum(sh, [])) == list(range(200))
+    loads = [sum(sd.race_cost(sfsgen.corpus_spec(200, i)) for i in s) for s in sh]
+    assert max(loads) / min(loads) < 1.02
+
+
+def test_expected_nnz_tracks_generator():
+    """The scheduling estimate is within ±25 % of the generated nnz for each corpus class."""
+    import sfsgen
+    for i in range(8):  # two of each class, small sizes only
+        sp = sfsgen.corpus_spec(200, i)
+        if sp.m > 200000:
+            continue
+        est, act = sd.expected_nnz(sp), sfsgen.generate(sp).nnz
+        assert 0.75 * act <= est <= 1.25 * act, (i, est, act)
