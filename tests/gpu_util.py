@@ -61,16 +61,20 @@ def check_spmv(A, fmt, M: sfs.Matrix, x: np.ndarray, dtype: int, ctx=""):
     """Per-row |y_gpu - y_ref| <= tol * (|A||x|)_r; rows with (|A||x|)_r = 0 must give exactly 0."""
     import torch
     xd = torch.from_numpy(x).cuda()
-    y = torch.full((A.m,), float("nan"), dtype=xd.dtype, device="cuda")
-    sfs.spmv(fmt, M, xd, y)
-    torch.cuda.synchronize()
-    yg = y.cpu().numpy().astype(np.float64)
     yr, ay = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val.astype(np.float64), x.astype(np.float64))
     tol = TOL[dtype]
-    err = np.abs(yg - yr)
-    bad = ~(err <= tol * ay)
-    zero_rows = ay == 0
-    bad |= zero_rows & (yg != 0)
-    assert not bad.any(), (f"{ctx} {sfs.FORMAT_NAMES[fmt]}: {int(bad.sum())} rows out of tolerance; first "
-                           f"{np.nonzero(bad)[0][:5]} gpu {yg[bad][:5]} ref {yr[bad][:5]} |A||x| {ay[bad][:5]}")
+    # twice, y poisoned with NaN before each call: every row must be written, and the kernels' carry
+    # flags must be back to their initial state after a call
+    for rep in range(2):
+        y = torch.full((A.m,), float("nan"), dtype=xd.dtype, device="cuda")
+        sfs.spmv(fmt, M, xd, y)
+        torch.cuda.synchronize()
+        yg = y.cpu().numpy().astype(np.float64)
+        err = np.abs(yg - yr)
+        bad = ~(err <= tol * ay)
+        zero_rows = ay == 0
+        bad |= zero_rows & (yg != 0)
+        assert not bad.any(), (f"{ctx} {sfs.FORMAT_NAMES[fmt]} call {rep}: {int(bad.sum())} rows out of tolerance; "
+                               f"first {np.nonzero(bad)[0][:5]} gpu {yg[bad][:5]} ref {yr[bad][:5]} "
+                               f"|A||x| {ay[bad][:5]}")
     return yg

@@ -230,7 +230,7 @@ def test_launch_count_increases():
     c0 = sfs.launch_count()
     for _ in range(3):
         sfs.spmv(sfs.COO, M, x, y)
-    assert sfs.launch_count() - c0 == 6  # memset + kernel per COO SpMV
+    assert sfs.launch_count() - c0 == 6  # zero kernel + COO kernel per COO SpMV
 
 
 def _tile_edge_csr(dtype, cap=None):
@@ -277,6 +277,10 @@ def test_csr_tile_edges(dtype, cap):
     assert M.layout().variant == 3
     check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="tile-edges")
     M.free()
+    # the same rows through the one-launch COO kernel (gaps, split rows, a row over ~1000 warp ranges)
+    M = sfs.convert(dA, sfs.COO)
+    check_spmv(A, sfs.COO, M, x, A.dtype, ctx="coo-edges")
+    M.free()
     # borrowed arrays that are not 32 B aligned (a view at an element offset): scalar-load path
     t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
     colb = torch.empty(A.nnz + 1, dtype=torch.int32, device="cuda")
@@ -287,3 +291,40 @@ def test_csr_tile_edges(dtype, cap):
     M = sfs.convert(dB, sfs.CSR, sfs.default_opts(csr_variant=3))
     check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="tile-edges-misaligned")
     M.free()
+
+
+@pytest.mark.parametrize("shape", ["one_row", "two_rows", "first_last", "diag_gaps"])
+def test_split_rows_and_gaps(shape):
+    """Row layouts that exercise the carries of the one-launch COO and CSR tile kernels: one row holding
+    every entry (all warps but the first are middle pieces), two long rows meeting mid-range, entries only
+    in the first and last rows (one long run of empty rows), and a sparse diagonal (gaps everywhere)."""
+    rng = np.random.default_rng(5)
+    m, n = 40_000, 3_000_000
+    lens = np.zeros(m, np.int64)
+    if shape == "one_row":
+        lens[m // 2] = 2_000_000
+    elif shape == "two_rows":
+        lens[7] = 1_234_567
+        lens[8] = 1_000_003
+    elif shape == "first_last":
+        lens[0] = 700_001
+        lens[-1] = 900_000
+    else:
+        lens[::3] = 1
+        lens[5] = 1_500_000
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    z = int(rp[-1])
+    col = np.empty(z, np.int64)
+    for r in np.nonzero(lens)[0]:
+        L = int(lens[r])
+        col[rp[r]:rp[r + 1]] = np.sort(rng.choice(n, L, replace=False)) if L > 1 else [r % n]
+    val = rng.uniform(0.5, 1.0, z) * rng.choice([-1.0, 1.0], z)
+    A = sfsgen.CSR(m, n, rp.astype(np.int32), col.astype(np.int32), val)
+    x = sfsgen.vector(3, n, A.dtype)
+    dA = to_dev(A)
+    for fmt, opts in [(sfs.CSR, sfs.default_opts(csr_variant=3)), (sfs.CSR, sfs.default_opts(csr_variant=1)),
+                      (sfs.COO, None)]:
+        M = sfs.convert(dA, fmt, opts)
+        check_spmv(A, fmt, M, x, A.dtype, ctx=f"{shape}/{sfs.FORMAT_NAMES[fmt]}")
+        M.free()
