@@ -50,6 +50,8 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--out", default=None, help="also append the JSON line to this file")
     p.add_argument("--dump", default=None, help="write per-matrix results of the last timed step (JSONL)")
+    p.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                   help="gloo: host-side collectives, lets N ranks share one GPU (tests of the N > 1 path only)")
     return p.parse_args()
 
 
@@ -213,10 +215,16 @@ def run_ours(args):
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
 
     rank, world, local = dist_env()
+    local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
+    gloo = args.dist_backend == "gloo"
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if gloo:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
+    cdev = torch.device("cpu") if gloo else dev  # where the collectives' tensors live
     stream = torch.cuda.current_stream()
 
     host = generate_host(corpus_ids(rank, args.corpus, world))
@@ -229,11 +237,11 @@ def run_ours(args):
     n = len(mats)
     n_max = n
     if world > 1:  # LPT shards differ by a matrix or two: pad the gathered result rows
-        nt = torch.tensor([n], dtype=torch.int64, device=dev)
+        nt = torch.tensor([n], dtype=torch.int64, device=cdev)
         dist.all_reduce(nt, op=dist.ReduceOp.MAX)
         n_max = int(nt.item())
-    gather_buf = torch.full((n_max * 9,), -1.0, dtype=torch.float64, device=dev)
-    all_buf = torch.zeros(world * n_max * 9, dtype=torch.float64, device=dev)
+    gather_buf = torch.full((n_max * 9,), -1.0, dtype=torch.float64, device=cdev)
+    all_buf = torch.zeros(world * n_max * 9, dtype=torch.float64, device=cdev)
 
     def step(batch):
         feats, labs = sfs.label_corpus(batch, opts)
@@ -252,14 +260,14 @@ def run_ours(args):
     def maxr(v):
         if world == 1:
             return v
-        tt = torch.tensor([v], dtype=torch.float64, device=dev)
+        tt = torch.tensor([v], dtype=torch.float64, device=cdev)
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         return float(tt.item())
 
     def sumr(v):
         if world == 1:
             return v
-        tt = torch.tensor([v], dtype=torch.float64, device=dev)
+        tt = torch.tensor([v], dtype=torch.float64, device=cdev)
         dist.all_reduce(tt, op=dist.ReduceOp.SUM)
         return float(tt.item())
 

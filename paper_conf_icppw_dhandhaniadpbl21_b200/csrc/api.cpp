@@ -399,7 +399,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       void* cv = own(sv * std::max(nc, 1LL));
       if (!ec || !ev || !cr || !cc || !cv) return bail(SFS_ERR_OOM, "hyb");
       TRY_CUDA(launch_csr2ell(d.dtype, d.rp, d.col, d.val, m, P, (int)K, ec, ev, s));
-      // rows overflowing by <= kHybRowwiseMax: keep the per-row overflow offsets for the one-launch SpMV
+      // rows overflowing by <= 32 (64 below 2^20 nnz): keep the per-row overflow offsets for the one-launch SpMV
       A->variant = hyb_rowwise(f.nnz_max, K, nc, z);
       if (nc > 0) {
         Temps t(s);

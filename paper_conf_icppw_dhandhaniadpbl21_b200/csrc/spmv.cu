@@ -27,6 +27,7 @@
 //                S slot-parts per row group; HYB = ELL part (writes y) then COO part (accumulates).
 //   DIA        : 4 (fp64) / 8 (fp32) rows per thread 256 apart (coalesced slab and x), S diagonal
 //                parts per row block.
+#include <stdio.h>
 #include <stdlib.h>
 
 #include "common.cuh"
@@ -724,10 +725,11 @@ constexpr int kEllThreads = 256;
 template <typename T> constexpr int ell_batch() { return sizeof(T) == 4 ? 8 : 4; }   // bytes in flight per thread
 template <typename T> constexpr int ell_ctas() { return sizeof(T) == 4 ? 3 : 4; }    // CTAs / SM (register cap)
 
-// OVF (HYB whose rows overflow the ELL part by at most kHybRowwiseMax entries): part 0 of each row
-// group also adds its rows' COO-part entries, located by the per-row overflow offsets ovf[0..m]
-// kept from the conversion -- HYB in one launch, y written once.
-constexpr long long kHybRowwiseMax = 32;
+// OVF (HYB whose rows overflow the ELL part by at most kHybRowwiseLarge / kHybRowwiseSmall entries):
+// the parts of each row group also add its rows' COO-part entries, located by the per-row overflow
+// offsets ovf[0..m] kept from the conversion -- HYB in one launch, y written once.
+constexpr long long kHybRowwiseSmall = 64;  // z < 2^20 (latency-bound sizes)
+constexpr long long kHybRowwiseLarge = 32;
 
 template <typename T, bool OVF>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
@@ -755,7 +757,7 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
     acc_t acc[4] = {0, 0, 0, 0};
     if (grp < groups) {
       int ob[5];
-      if (OVF && p == 0) {
+      if (OVF) {
 #pragma unroll
         for (int q = 0; q <= 4; q++) ob[q] = __ldg(ovf + (r + q < m ? r + q : m));
       }
@@ -787,9 +789,10 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
         if (c.z >= 0) acc[2] += (acc_t)v.v[2] * (acc_t)ld_x(x + c.z);
         if (c.w >= 0) acc[3] += (acc_t)v.v[3] * (acc_t)ld_x(x + c.w);
       }
-      if (OVF && p == 0) {
-        // the 4 rows' overflow entries are contiguous: [ob[0], ob[4]), 4 at a time, clamped loads
-        for (int k = ob[0]; k < ob[4]; k += 4) {
+      if (OVF) {
+        // the 4 rows' overflow entries are contiguous: [ob[0], ob[4]); batches of 4 (clamped loads),
+        // batch b taken by slot-part b mod S, so the parts share the walk
+        for (int k = ob[0] + 4 * p; k < ob[4]; k += 4 * S) {
           int c[4];
           T v[4];
 #pragma unroll
@@ -1150,12 +1153,21 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
   return cudaGetLastError();
 }
 
-// One-launch HYB when the overflow per row is short: <= 4 entries at any size, <= 32 below 2^20 nnz
-// (latency-bound sizes, where the second kernel's launch edge dominates).  Measured on corpus-200:
-// longer serial overflow walks lose to the COO kernel on large random-column matrices.
+// One-launch HYB when the overflow per row is short: <= 32 entries (<= 64 below 2^20 nnz), the walk
+// shared by the slot-parts.  Measured on 50 corpus-200 matrices with a COO part (tools/hyb_ab.sh,
+// profiles/r01/csr_variants.txt): HYB race time -4.8 % against the previous rule (<= 4, or <= 32
+// below 2^20) and -10 % against always two kernels; rows overflowing by thousands (power-law) keep
+// the ELL-part -> COO-part pair.
 int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) {
   const long long o = nnz_max - K;
-  return coo_nnz > 0 && (o <= 4 || (z < (1LL << 20) && o <= kHybRowwiseMax));
+  static long long small = -2, large = -2;  // SFS_HYB_ROWWISE="small,large": A/B overrides of the limits
+  if (small == -2) {
+    small = kHybRowwiseSmall;
+    large = kHybRowwiseLarge;
+    const char* e = getenv("SFS_HYB_ROWWISE");
+    if (e) sscanf(e, "%lld,%lld", &small, &large);
+  }
+  return coo_nnz > 0 && (o <= large || (z < (1LL << 20) && o <= small));
 }
 
 int spmv_kernels_per_call(const Matrix* A) {

@@ -78,3 +78,30 @@ def test_sharded_corpus_driver_single_rank():
         fo = oracle.features(A.m, A.n, A.rp, A.col)
         assert r["features"]["nnz"] == fo["nnz"] and r["features"]["nnz_sig"] == fo["nnz_sig"]
         assert 0 <= r["label"] < 5 and r["matrix_status"] == 0
+
+
+def test_bench_two_ranks_share_one_gpu():
+    """bench.py's N > 1 path end to end (LPT weak shards, result all-gather, max-over-ranks timing,
+    summed launch counts): torchrun with 2 ranks on this one GPU, gloo collectives on host tensors."""
+    import json
+    import os
+    import socket
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(root, "bench.py"),
+           "--gpus", "2", "--steps", "1", "--warmup", "1", "--corpus", "6", "--e2e-steps", "1",
+           "--no-cpu-baseline", "--dist-backend", "gloo"]
+    r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["config"]["matrices_all_ranks"] == 12
+    assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
+    assert d["scaling"] == "weak"

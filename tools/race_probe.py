@@ -12,6 +12,7 @@ def main():
     ap.add_argument("--rounds", type=int, default=3)
     ap.add_argument("--tag", default=os.path.basename(os.environ.get("SFS_LIB", "libsfs.so")))
     ap.add_argument("--json", default=None)
+    ap.add_argument("--quiet", action="store_true")
     a = ap.parse_args()
     import torch
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
@@ -30,12 +31,13 @@ def main():
         cur = [L["t_spmv_us"] for L in labs]
         best = cur if best is None else [[min(p, q) for p, q in zip(b, c)] for b, c in zip(best, cur)]
     tot = [sum(r[f] for r in best) for f in range(5)]
-    print(a.tag, "total", [round(v, 1) for v in tot])
-    for i, M, r in zip(ids, mats, best):
-        print(f"  {i:4d} nnz={M.nnz:9d}", " ".join(f"{sfs.FORMAT_NAMES[f]}:{r[f]:7.2f}" for f in range(5)))
     if a.json:
         with open(a.json, "a") as fh:
             fh.write(json.dumps({"tag": a.tag, "ids": ids, "t": best}) + "\n")
+    print(a.tag, "total", [round(v, 1) for v in tot], flush=True)
+    if not a.quiet:
+        for i, M, r in zip(ids, mats, best):
+            print(f"  {i:4d} nnz={M.nnz:9d}", " ".join(f"{sfs.FORMAT_NAMES[f]}:{r[f]:7.2f}" for f in range(5)))
 
 
 if __name__ == "__main__":
