@@ -353,13 +353,15 @@ def run_ours(args):
     launches_dom = sum(1 for L in labs if L["status"][sfs.FORMAT_NAMES.index(dom)] == 0) * args.reps
     bytes_per_launch = (per_fmt[dom]["gbs"] * 1e9 * per_fmt[dom]["spmv_time_s"] / launches_dom) if launches_dom else 0
     traffic, traffic_src = None, None
-    try:
-        with open(os.path.join(ROOT, "profiles", "traffic.json")) as fh:
+    try:  # ncu dram__bytes_read+write of this format's kernels on this workload, hot reps (tools/traffic_corpus.py)
+        with open(os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json")) as fh:
             tj = json.load(fh).get(dom)
-        if tj:  # measured DRAM/algorithmic ratio of this format's kernel (ncu --set full, cold, configs[3])
+        if tj:
             traffic = tj["ratio"] * bytes_per_launch
-            traffic_src = (f"dram__bytes_read+write / algorithmic = {tj['ratio']:.3f} for {tj['kernel']} "
-                           f"(profiles/traffic.json), times the mean algorithmic bytes per launch")
+            traffic_src = (f"ncu dram__bytes_read.sum + dram__bytes_write.sum of {tj['kernel']} over the corpus-200 race "
+                           f"(last of 2 back-to-back calls per matrix, --cache-control none) = {tj['ratio']:.3f} x "
+                           f"the algorithmic bytes (profiles/r01/traffic_corpus200.json); < 1: the hot reps re-read "
+                           f"part of each matrix from L2")
     except Exception:
         pass
     step_time = t_dev / args.steps
