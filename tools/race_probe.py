@@ -13,6 +13,7 @@ def main():
     ap.add_argument("--tag", default=os.path.basename(os.environ.get("SFS_LIB", "libsfs.so")))
     ap.add_argument("--json", default=None)
     ap.add_argument("--quiet", action="store_true")
+    ap.add_argument("--csr-variant", type=int, default=-1)
     a = ap.parse_args()
     import torch
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
@@ -24,7 +25,7 @@ def main():
         sp = sfsgen.corpus_spec(200, i)
         A = sfsgen.generate(sp)
         mats.append(sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), t(sfsgen.vector(sp.seed, A.n, A.dtype))))
-    opts = sfs.default_opts(formats_mask=a.mask)
+    opts = sfs.default_opts(formats_mask=a.mask, csr_variant=a.csr_variant)
     best = None
     for _ in range(a.rounds):
         _, labs = sfs.label_corpus(mats, opts)
