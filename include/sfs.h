@@ -154,6 +154,13 @@ sfs_status sfs_spmv(sfs_format f, sfs_matrix A, const void *x, void *y, void *st
 sfs_status sfs_label_corpus(const sfs_csr *mats, int64_t n, const sfs_race_opts *opt, sfs_features_t *feats,
                             sfs_label_t *labels, void *stream);
 
+/* Halo send buffer of the row-partitioned SpMV (y = A·x of P:L31 split by
+   rows): dst[i] = src[idx[i]] for 0 <= i < n.  src: the rank's slice of x (device, dtype); idx: int32
+   device array of local indices, each in [0, len(src)) (not checked); dst: n entries (device, dtype),
+   caller-owned.  Asynchronous on `stream`, one kernel launch (none if n == 0).  INVALID_ARG for a bad
+   dtype, n < 0 or a null pointer with n > 0. */
+sfs_status sfs_gather(sfs_dtype dtype, const void *src, const int32_t *idx, int64_t n, void *dst, void *stream);
+
 sfs_status sfs_matrix_free(sfs_matrix A); /* stream-ordered on the stream it was created on */
 sfs_status sfs_matrix_describe(sfs_matrix A, sfs_layout_t *out);
 

@@ -94,6 +94,7 @@ def lib():
         L.sfs_features.argtypes = [ctypes.POINTER(CsrStruct), ctypes.POINTER(RaceOpts), ctypes.POINTER(FeaturesStruct), _P]
         L.sfs_convert.argtypes = [ctypes.POINTER(CsrStruct), _I32, ctypes.POINTER(RaceOpts), ctypes.POINTER(_P), _P]
         L.sfs_spmv.argtypes = [_I32, _P, _P, _P, _P]
+        L.sfs_gather.argtypes = [_I32, _P, _P, _I64, _P, _P]
         L.sfs_label_corpus.argtypes = [ctypes.POINTER(CsrStruct), _I64, ctypes.POINTER(RaceOpts),
                                        ctypes.POINTER(FeaturesStruct), ctypes.POINTER(LabelStruct), _P]
         L.sfs_matrix_free.argtypes = [_P]
@@ -238,6 +239,14 @@ def spmv(fmt: int, A: Matrix, x, y, stream=None):
     """y = A x on the GPU (sfs_spmv); asynchronous on `stream`."""
     _check(lib().sfs_spmv(fmt, A.handle, x.data_ptr(), y.data_ptr(), _stream_ptr(stream)), "sfs_spmv")
     return y
+
+
+def gather(src, idx, dst, stream=None):
+    """dst[i] = src[idx[i]] on the GPU (sfs_gather): the halo send buffer of the row partition."""
+    dt = F64 if src.element_size() == 8 else F32
+    _check(lib().sfs_gather(dt, src.data_ptr(), idx.data_ptr(), idx.numel(), dst.data_ptr(), _stream_ptr(stream)),
+           "sfs_gather")
+    return dst
 
 
 def label_corpus(mats: Sequence[Csr], opts: Optional[RaceOpts] = None, stream=None):

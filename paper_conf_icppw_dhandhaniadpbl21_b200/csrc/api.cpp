@@ -586,6 +586,14 @@ sfs_status sfs_spmv(sfs_format f, sfs_matrix Ah, const void* x, void* y, void* s
   return SFS_OK;
 }
 
+sfs_status sfs_gather(sfs_dtype dtype, const void* src, const int32_t* idx, int64_t n, void* dst, void* stream) {
+  if (n < 0 || (n > 0 && (!src || !idx || !dst)) || (dtype != SFS_F32 && dtype != SFS_F64))
+    return fail(SFS_ERR_INVALID_ARG, "sfs_gather: bad argument");
+  cudaError_t e = launch_gather((int)dtype, src, idx, n, dst, (cudaStream_t)stream);
+  if (e != cudaSuccess) return cuda_fail(e, "gather launch");
+  return SFS_OK;
+}
+
 sfs_status sfs_matrix_free(sfs_matrix A) {
   matrix_free((Matrix*)A);
   return SFS_OK;

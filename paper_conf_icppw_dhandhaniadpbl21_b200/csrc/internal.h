@@ -103,6 +103,8 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
 int csr_vector_tpv(long long m, long long z);
 int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
+// dst[i] = src[idx[i]], i < n (exchange.cu: halo send buffers of the row-partitioned SpMV)
+cudaError_t launch_gather(int dtype, const void* src, const int* idx, long long n, void* dst, cudaStream_t s);
 cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s);
 
 // ---------------------------------------------------------------- semi-supervised predictor (cluster.cu)

@@ -8,8 +8,10 @@ The labelling pass shards in the two ways SURVEY §8(e) names:
    The paper labels one platform at a time (§5.1); sharding the M×F×N experiments of P:L46
    over GPUs is the build's addition.
 2. Row partition of one large matrix (one exchange per SpMV): rank k holds the contiguous row block
-   A[r_k:r_{k+1}, :] with global column ids; each SpMV is ``all_gather_into_tensor(x_full, x_local)``
-   followed by the local ``sfs_spmv``.
+   A[r_k:r_{k+1}, :]; each SpMV is either ``all_gather_into_tensor(x_full, x_local)`` followed by the
+   local ``sfs_spmv`` (global column ids), or -- SURVEY §8(f) f3 -- a halo exchange: only the ghost
+   entries of x the block references, point-to-point from their owners, into an extended vector the
+   block's columns were renumbered into (``halo_plan`` / ``rowpart_halo_iterate``).
 
 Everything that touches matrix data runs in libsfs; this module only partitions, launches and
 gathers.  The labeller / SpMV callables are injectable so the host logic is testable with gloo on CPU.
@@ -220,3 +222,171 @@ def rowpart_spmv_iterate(part: RowPartition, local_spmv: Callable, x_local, iter
         if swap:
             cur = y_local.clone()
     return y_local
+
+
+# ------------------------------------------------------------------ row partition with a halo exchange
+# instead of all-gathering all of x before every SpMV (every rank receives (P-1)/P of
+# x), each rank receives only the x entries its row block references outside its own slice -- its
+# ghost columns -- point-to-point from their owners.  For the 3D 27-point stencil (configs[3]) that is
+# two 128^2-row planes per neighbour instead of (P-1)/P of 2^21 rows.  The block's columns are renumbered
+# into an extended vector x_ext = [ghosts below r0 | own slice | ghosts at or above r1]; a contiguous
+# run of ghosts keeps its offsets, so a banded block stays banded (DIA admissible, same diagonals).
+# The SpMV writes y straight into the own-slice view of the next x_ext, the send buffer is packed by
+# sfs_gather, and the exchange is one batch of NCCL send/recv pairs.
+
+
+@dataclass
+class HaloPlan:
+    world: int
+    rank: int
+    r0: int
+    r1: int
+    lo: np.ndarray        # ghost columns < r0, ascending (global ids) -> x_ext[0 : n_lo]
+    hi: np.ndarray        # ghost columns >= r1, ascending -> x_ext[n_lo + n_local :]
+    recv: List[tuple]     # (source rank, offset in x_ext, count), ascending source
+    send: List[tuple]     # (destination rank, offset in the send buffer, count), ascending destination
+    send_idx: np.ndarray  # int32 indices into the own slice, concatenated by destination
+    col_ext: np.ndarray   # int32 columns of the row block renumbered into x_ext
+
+    @property
+    def n_local(self) -> int:
+        return self.r1 - self.r0
+
+    @property
+    def n_lo(self) -> int:
+        return len(self.lo)
+
+    @property
+    def n_ext(self) -> int:
+        return len(self.lo) + self.n_local + len(self.hi)
+
+    @property
+    def recv_count(self) -> int:
+        return len(self.lo) + len(self.hi)
+
+
+def halo_needs(part: RowPartition, col_block: np.ndarray):
+    """Ghost columns of a row block: the distinct columns outside the block's own slice [r0, r1)."""
+    b = part.bounds
+    r0, r1 = b[part.rank], b[part.rank + 1]
+    u = np.unique(np.asarray(col_block, dtype=np.int64))
+    return u[u < r0], u[u >= r1]
+
+
+def remap_columns(col_block: np.ndarray, r0: int, r1: int, lo: np.ndarray, hi: np.ndarray) -> np.ndarray:
+    c = np.asarray(col_block, dtype=np.int64)
+    out = np.empty_like(c)
+    below, own, above = c < r0, (c >= r0) & (c < r1), c >= r1
+    out[below] = np.searchsorted(lo, c[below])
+    out[own] = len(lo) + (c[own] - r0)
+    out[above] = len(lo) + (r1 - r0) + np.searchsorted(hi, c[above])
+    return out.astype(np.int32)
+
+
+def _segments(ids: np.ndarray, owner_block: int, base: int):
+    """(owner rank, offset, count) runs of an ascending id list, offsets from `base`."""
+    segs = []
+    if len(ids) == 0:
+        return segs
+    own = ids // owner_block
+    starts = np.flatnonzero(np.r_[True, own[1:] != own[:-1]])
+    ends = np.r_[starts[1:], len(ids)]
+    for s, e in zip(starts, ends):
+        segs.append((int(own[s]), base + int(s), int(e - s)))
+    return segs
+
+
+def build_halo_plan(part: RowPartition, col_block: np.ndarray, requests: Sequence[np.ndarray]) -> HaloPlan:
+    """The rank's plan, given `requests[j]` = the global columns rank j needs from this rank (ascending)."""
+    b = part.bounds
+    r0, r1 = b[part.rank], b[part.rank + 1]
+    lo, hi = halo_needs(part, col_block)
+    recv = _segments(lo, part.block, 0) + _segments(hi, part.block, len(lo) + (r1 - r0))
+    send, idx, off = [], [], 0
+    for j, req in enumerate(requests):
+        req = np.asarray(req, dtype=np.int64)
+        if j == part.rank or len(req) == 0:
+            continue
+        assert req.min() >= r0 and req.max() < r1, "request outside the owner's slice"
+        send.append((j, off, len(req)))
+        idx.append(req - r0)
+        off += len(req)
+    send_idx = (np.concatenate(idx) if idx else np.zeros(0, np.int64)).astype(np.int32)
+    return HaloPlan(part.world, part.rank, r0, r1, lo, hi, recv, send, send_idx,
+                    remap_columns(col_block, r0, r1, lo, hi))
+
+
+def halo_requests_by_owner(part: RowPartition, col_block: np.ndarray) -> List[np.ndarray]:
+    """What this rank needs from each rank (index j: the columns owned by rank j)."""
+    lo, hi = halo_needs(part, col_block)
+    g = np.concatenate([lo, hi])
+    own = g // part.block
+    return [g[own == j] for j in range(part.world)]
+
+
+def halo_plan(part: RowPartition, col_block: np.ndarray, group=None, device=None) -> HaloPlan:
+    """Collective (setup only): every rank tells each owner which of its columns it needs
+    (all_to_all_single of the counts, then of the ids), then builds its plan."""
+    import torch
+    import torch.distributed as dist
+    need = halo_requests_by_owner(part, col_block)
+    if part.world == 1:
+        return build_halo_plan(part, col_block, [np.zeros(0, np.int64)])
+    dev = device or "cpu"
+    cnt_out = torch.tensor([len(v) for v in need], dtype=torch.int64, device=dev)
+    cnt_in = torch.empty(part.world, dtype=torch.int64, device=dev)
+    dist.all_to_all_single(cnt_in, cnt_out, group=group)
+    cin = cnt_in.cpu().tolist()
+    ids_out = torch.from_numpy(np.concatenate(need).astype(np.int64)).to(dev)
+    ids_in = torch.empty(int(sum(cin)), dtype=torch.int64, device=dev)
+    dist.all_to_all_single(ids_in, ids_out, output_split_sizes=cin, input_split_sizes=[len(v) for v in need],
+                           group=group)
+    got = ids_in.cpu().numpy()
+    req, o = [], 0
+    for c in cin:
+        req.append(got[o:o + c])
+        o += c
+    return build_halo_plan(part, col_block, req)
+
+
+def halo_plans_local(m: int, n: int, world: int, col_blocks: Sequence[np.ndarray]) -> List[HaloPlan]:
+    """Every rank's plan built in one process (no collectives): the same plans halo_plan() builds, for
+    simulating the P ranks on one GPU and for tests."""
+    parts = [RowPartition(m, n, world, k) for k in range(world)]
+    needs = [halo_requests_by_owner(parts[k], col_blocks[k]) for k in range(world)]
+    return [build_halo_plan(parts[k], col_blocks[k], [needs[j][k] for j in range(world)]) for k in range(world)]
+
+
+def rowpart_halo_iterate(plan: HaloPlan, local_spmv: Callable, gather: Callable, x_local, iters: int,
+                         group=None, ranks: Optional[Sequence[int]] = None):
+    """`iters` power-iteration steps y_k = A_k x on the halo plan: exchange ghosts, SpMV into the own
+    slice of the other x_ext buffer.  `local_spmv(x_ext, y_view)` runs the rank's remapped block (sfs_spmv
+    on a GPU); `gather(x_own_view, idx_tensor, out)` packs the send buffer (sfs_gather).  `ranks`: group
+    ranks of the partition's ranks (default: identity).  Returns the final own slice (a view)."""
+    import torch
+    import torch.distributed as dist
+    dev, dt = x_local.device, x_local.dtype
+    xa = torch.zeros(plan.n_ext, dtype=dt, device=dev)
+    xb = torch.zeros(plan.n_ext, dtype=dt, device=dev)
+    own = slice(plan.n_lo, plan.n_lo + plan.n_local)
+    xa[own].copy_(x_local)
+    idx = torch.from_numpy(plan.send_idx.astype(np.int32)).to(dev)
+    sbuf = torch.empty(len(plan.send_idx), dtype=dt, device=dev)
+    gr = (lambda k: k) if ranks is None else (lambda k: ranks[k])
+
+    def exchange(buf):
+        if plan.world == 1 or (not plan.send and not plan.recv):
+            return
+        gather(buf[own], idx, sbuf)
+        ops = [dist.P2POp(dist.isend, sbuf[o:o + c], gr(j), group=group) for j, o, c in plan.send]
+        ops += [dist.P2POp(dist.irecv, buf[o:o + c], gr(j), group=group) for j, o, c in plan.recv]
+        for r in dist.batch_isend_irecv(ops):
+            r.wait()
+
+    cur, nxt = xa, xb
+    exchange(cur)
+    for _ in range(iters):
+        local_spmv(cur, nxt[own])
+        exchange(nxt)
+        cur, nxt = nxt, cur
+    return cur[own]

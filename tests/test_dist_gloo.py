@@ -153,3 +153,99 @@ def test_expected_nnz_tracks_generator():
             continue
         est, act = sd.expected_nnz(sp), sfsgen.generate(sp).nnz
         assert 0.75 * act <= est <= 1.25 * act, (i, est, act)
+
+
+def _halo_case(kind):
+    import sfsgen
+    from helpers import random_csr
+    if kind == "stencil":
+        return sfsgen.stencil3d27(12)
+    rng = np.random.default_rng(9)
+    return random_csr(rng, 1500, 1500, 0.01, empty_rows=0.1, dense_rows=1)
+
+
+@pytest.mark.parametrize("kind", ["stencil", "random"])
+@pytest.mark.parametrize("world", [1, 3, 4])
+def test_halo_plans_reproduce_the_row_blocks(kind, world):
+    """Every rank's renumbered block applied to x_ext = [x[lo] | own slice | x[hi]] gives its rows of A·x
+    exactly as the global-column block does; rank j sends rank k exactly the ghosts k receives from j;
+    a stencil block keeps its diagonals (contiguous ghost runs keep offsets)."""
+    import oracle
+    A = _halo_case(kind)
+    x = np.random.default_rng(1).uniform(-1, 1, A.n)
+    blocks = []
+    for k in range(world):
+        b = sd.row_blocks(A.m, world)
+        blocks.append(sd.slice_rows(A.rp, A.col, A.val, b[k], b[k + 1]))
+    plans = sd.halo_plans_local(A.m, A.n, world, [c for _, c, _ in blocks])
+    yg, _ = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
+    for k, (P, (rp, col, val)) in enumerate(zip(plans, blocks)):
+        xe = np.concatenate([x[P.lo], x[P.r0:P.r1], x[P.hi]])
+        assert P.n_ext == len(xe) and P.col_ext.max(initial=-1) < P.n_ext and P.col_ext.min(initial=0) >= 0
+        y, _ = oracle.spmv_csr(len(rp) - 1, P.n_ext, rp, P.col_ext, val, xe)
+        assert np.array_equal(y, yg[P.r0:P.r1])  # same entries in the same order: bitwise
+        for j, o, c in P.recv:  # what k receives from j is what j packs for k
+            Q = plans[j]
+            so = [(oo, cc) for d, oo, cc in Q.send if d == k]
+            assert len(so) == 1 and so[0][1] == c
+            got = Q.send_idx[so[0][0]:so[0][0] + c] + Q.r0
+            want = np.concatenate([P.lo, P.hi])[o - (0 if o < P.n_lo else P.n_local):][:c]
+            assert np.array_equal(got, want)
+        if kind == "stencil":
+            d_glob = np.unique(col.astype(np.int64) - np.repeat(np.arange(P.r0, P.r1), np.diff(rp)))
+            d_ext = np.unique(P.col_ext.astype(np.int64) - P.n_lo - np.repeat(np.arange(P.n_local), np.diff(rp)))
+            assert np.array_equal(d_glob, d_ext)
+
+
+def _halo_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        A = _halo_case("stencil")
+        part = sd.RowPartition(A.m, A.n, world, rank)
+        b = part.bounds
+        rp, col, val = sd.slice_rows(A.rp, A.col, A.val, b[rank], b[rank + 1])
+        plan = sd.halo_plan(part, col)  # collective: all_to_all of the requests
+
+        def local_spmv(xe, y):
+            yy, _ = oracle.spmv_csr(len(rp) - 1, plan.n_ext, rp, plan.col_ext, val, xe.numpy())
+            y.copy_(torch.from_numpy(yy))
+
+        def gather(src, idx, out):
+            out.copy_(src[idx.long()])
+
+        x = torch.from_numpy(np.random.default_rng(2).uniform(-1, 1, A.n))
+        y = sd.rowpart_halo_iterate(plan, local_spmv, gather, x[b[rank]:b[rank + 1]].clone(), iters=3)
+        q.put((rank, y.numpy().copy(), plan.recv_count))
+    except Exception:
+        import traceback
+        q.put((rank, "ERROR", traceback.format_exc()))
+        raise
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_halo_exchange_power_iteration():
+    """Two ranks exchange only their ghost planes (batch_isend_irecv) and reproduce the global power
+    iteration; each receives one 12^2 plane instead of half of x."""
+    import oracle
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_halo_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = sorted([q.get(timeout=240) for _ in range(world)], key=lambda t: t[0])
+    for o in out:
+        assert not isinstance(o[1], str), o[2]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    A = _halo_case("stencil")
+    x = np.random.default_rng(2).uniform(-1, 1, A.n)
+    for _ in range(3):
+        x, _ = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
+    assert np.array_equal(np.concatenate([out[0][1], out[1][1]]), x)
+    assert out[0][2] == out[1][2] == 12 * 12

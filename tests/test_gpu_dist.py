@@ -105,3 +105,68 @@ def test_bench_two_ranks_share_one_gpu():
     assert d["n_gpus"] == 2 and d["config"]["matrices_all_ranks"] == 12
     assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
     assert d["scaling"] == "weak"
+
+
+def test_gather_kernel():
+    import torch
+    rng = np.random.default_rng(3)
+    for dt in (np.float64, np.float32):
+        src = rng.uniform(-1, 1, 100_003).astype(dt)
+        idx = rng.integers(0, len(src), 77_777).astype(np.int32)
+        s, i = torch.from_numpy(src).cuda(), torch.from_numpy(idx).cuda()
+        out = torch.empty(len(idx), dtype=s.dtype, device="cuda")
+        sfs.gather(s, i, out)
+        assert np.array_equal(out.cpu().numpy(), src[idx])
+    empty = torch.empty(0, dtype=torch.int32, device="cuda")
+    sfs.gather(s, empty, torch.empty(0, dtype=s.dtype, device="cuda"))  # n = 0: no launch, OK
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+@pytest.mark.parametrize("fmt", [sfs.CSR, sfs.DIA, sfs.ELL])
+def test_halo_exchange_power_iteration_simulated(world, fmt):
+    """SURVEY §8(f) f3 on one GPU: the P ranks' renumbered row blocks through sfs_convert / sfs_spmv, the
+    send buffers packed by sfs_gather and the point-to-point exchange done by device copies between the
+    simulated ranks; 3 power-iteration steps == the oracle's global iteration within tolerance.  DIA of
+    a stencil block keeps its 27 diagonals after the renumbering."""
+    import torch
+    A = sfsgen.generate(sfsgen.make_spec(sfsgen.ST3D27, ia=24))
+    x0 = sfsgen.vector(11, A.n)
+    b = sd.row_blocks(A.m, world)
+    blocks = [sd.slice_rows(A.rp, A.col, A.val, b[k], b[k + 1]) for k in range(world)]
+    plans = sd.halo_plans_local(A.m, A.n, world, [c for _, c, _ in blocks])
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    mats, bufs = [], []
+    for k, (P, (rp, _, val)) in enumerate(zip(plans, blocks)):
+        Ak = sfs.Csr(P.n_local, P.n_ext, t(rp), t(P.col_ext), t(val))
+        if fmt == sfs.DIA:
+            assert sfs.features(Ak)["diagonals"] == 27
+        mats.append(sfs.convert(Ak, fmt))
+        xa = torch.zeros(P.n_ext, dtype=torch.float64, device="cuda")
+        xa[P.n_lo:P.n_lo + P.n_local] = t(x0[P.r0:P.r1])
+        bufs.append([xa, torch.zeros_like(xa), t(P.send_idx.astype(np.int32)),
+                     torch.empty(len(P.send_idx), dtype=torch.float64, device="cuda")])
+
+    def exchange(which):
+        for k, P in enumerate(plans):
+            src = bufs[k][which]
+            sfs.gather(src[P.n_lo:P.n_lo + P.n_local], bufs[k][2], bufs[k][3])
+        for k, P in enumerate(plans):  # k receives from j: j's send segment addressed to k
+            for j, o, c in P.recv:
+                Q = plans[j]
+                (so,) = [oo for d, oo, cc in Q.send if d == k]
+                bufs[k][which][o:o + c] = bufs[j][3][so:so + c]
+
+    cur = 0
+    exchange(cur)
+    for _ in range(3):
+        for k, P in enumerate(plans):
+            sfs.spmv(fmt, mats[k], bufs[k][cur], bufs[k][1 - cur][P.n_lo:P.n_lo + P.n_local])
+        exchange(1 - cur)
+        cur = 1 - cur
+    y = np.concatenate([bufs[k][cur][P.n_lo:P.n_lo + P.n_local].cpu().numpy() for k, P in enumerate(plans)])
+    x = x0
+    for _ in range(3):
+        x, ax = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
+    assert np.all(np.abs(y - x) <= 1e-11 * (np.abs(x) + ax))
+    for M in mats:
+        M.free()

@@ -1,5 +1,6 @@
 #!/usr/bin/env python
-"""configs[3]: 3D 27-point stencil on 128^3 row-partitioned over N GPUs with an NCCL all-gather of x.
+"""configs[3]: 3D 27-point stencil on 128^3 row-partitioned over N GPUs: an NCCL all-gather of x, or
+(--exchange halo) NCCL send/recv of the ghost planes only.
 
     python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 tools/bench_rowpart.py
 
@@ -25,6 +26,7 @@ def main():
     ap.add_argument("--dtype", default="f64")
     ap.add_argument("--iters", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo"])
     args = ap.parse_args()
 
     import torch
@@ -45,7 +47,9 @@ def main():
     b = part.bounds
     rp, col, val = sd.slice_rows(A.rp, A.col, A.val, b[rank], b[rank + 1])
     t = lambda a: torch.from_numpy(a).cuda()
-    Ak = sfs.Csr(part.local_rows, A.n, t(rp), t(col), t(val))
+    halo = args.exchange == "halo"
+    plan = sd.halo_plan(part, col, device=torch.device("cuda", local)) if halo else None
+    Ak = sfs.Csr(part.local_rows, plan.n_ext if halo else A.n, t(rp), t(plan.col_ext if halo else col), t(val))
     fmt = sfs.FORMAT_NAMES.index(args.fmt)
     M = sfs.convert(Ak, fmt)
     feats = sfs.features(Ak)
@@ -53,7 +57,11 @@ def main():
     xs = torch.from_numpy(sfsgen.vector(5, A.n, dt)).cuda()
     x_local = xs[b[rank]:b[rank + 1]].clone()
     spmv = lambda xf, yl: sfs.spmv(fmt, M, xf, yl)
-    sd.rowpart_spmv_iterate(part, spmv, x_local, iters=args.warmup)
+    if halo:
+        iterate = lambda it: sd.rowpart_halo_iterate(plan, spmv, sfs.gather, x_local, iters=it)
+    else:
+        iterate = lambda it: sd.rowpart_spmv_iterate(part, spmv, x_local, iters=it)
+    iterate(args.warmup)
 
     def timed(fn):
         if world > 1:
@@ -69,7 +77,7 @@ def main():
             dist.all_reduce(v, op=dist.ReduceOp.MAX)
         return float(v.item())
 
-    t_iter = timed(lambda: sd.rowpart_spmv_iterate(part, spmv, x_local, iters=args.iters)) / args.iters
+    t_iter = timed(lambda: iterate(args.iters)) / args.iters
     blk = part.block
     xp = torch.zeros(blk, dtype=xs.dtype, device="cuda")
     xf = torch.empty(blk * world, dtype=xs.dtype, device="cuda")
@@ -82,9 +90,11 @@ def main():
             else:
                 xf.copy_(xp)
 
+    xm = torch.zeros(plan.n_ext, dtype=xs.dtype, device="cuda") if halo else xs
+
     def mv():
         for _ in range(args.iters):
-            spmv(xs, yl)
+            spmv(xm, yl)
 
     t_ag = timed(ag) / args.iters
     t_mv = timed(mv) / args.iters
@@ -93,7 +103,9 @@ def main():
         dist.all_reduce(tot_bytes)
     if rank == 0:
         print(json.dumps({"config": f"configs[3] 3D27 {args.N}^3 {args.dtype} row-partitioned", "n_gpus": world,
-                          "format": args.fmt, "t_iter_us": t_iter * 1e6, "t_allgather_us": t_ag * 1e6,
+                          "format": args.fmt, "exchange": args.exchange, "t_iter_us": t_iter * 1e6,
+                          "t_allgather_us": t_ag * 1e6,
+                          "halo_recv_entries_rank0": plan.recv_count if halo else None,
                           "t_spmv_us": t_mv * 1e6, "agg_spmv_gbs": float(tot_bytes.item()) / t_iter / 1e9,
                           "rows_per_rank": part.block}))
     if world > 1:
