@@ -408,8 +408,10 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
   pdl_early();
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < tiles; t += (long long)gridDim.x * blockDim.x) {
     const int r = carry_row[t];
-    const acc_t v = carry_val[t];
-    if (r < m && v != 0) atomicAdd(y + r, (T)v);
+    if (r < m) {  // carry_val is only written for a carried row
+      const acc_t v = carry_val[t];
+      if (v != 0) atomicAdd(y + r, (T)v);
+    }
   }
   pdl_trigger();
 }
