@@ -346,7 +346,8 @@ def run_ours(args):
     peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
     if not peak:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
-    kernels = {"CSR": "k_spmv_csr_stream (regular rows) / k_spmv_csr_merge + fixup (skewed rows)",
+    kernels = {"CSR": "k_spmv_csr_tile<bitmap> + fixup (large or skewed, no empty rows) / k_spmv_csr_stream "
+                      "(small regular) / k_spmv_csr_merge + fixup (many empty rows)",
                "COO": "k_zero + k_spmv_coo", "ELL": "k_spmv_ell", "HYB": "k_spmv_ell + k_spmv_coo<ACCUM>",
                "DIA": "k_spmv_dia"}
     achieved = per_fmt[dom]["gbs"]

@@ -77,7 +77,8 @@ typedef struct {
   uint32_t admissible_mask; /* bit f set iff format f is admissible (Q11) */
   int32_t csr_variant;      /* CSR kernel the library picks for this matrix (Q17): 0 vector (CUSP
                                mapping), 1 merge path, 2 stream (warp per 32 rows), 3 tile
-                               (nnz-balanced 256-entry chunks, rows rebuilt from row_ptr) */
+                               (nnz-balanced 256-entry chunks, rows rebuilt from row_ptr), 4 tile
+                               with rows from a row-start bitmap (no empty rows) */
 } sfs_features_t;
 
 typedef struct sfs_matrix_ *sfs_matrix; /* opaque, library-owned */
@@ -108,7 +109,7 @@ typedef struct {
   int64_t fill_slack;    /* (1<<20) */
   double hyb_rel_speed;  /* Q6 HYB width rule (3.0) */
   int64_t hyb_breakeven; /* (4096) */
-  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream; 3 = tile */
+  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream; 3 = tile; 4 = tile with row ids from a row-start bitmap (falls back to 3 when a row is empty) */
   int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (0: direct launches with PDL) */
 } sfs_race_opts;
 

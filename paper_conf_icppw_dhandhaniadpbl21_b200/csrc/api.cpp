@@ -180,13 +180,14 @@ static void finalize(long long m, long long n, long long z, const DevAggr& a, lo
   f->admissible_mask = mask;
   // Q17 (measured on corpus-200): merge path when empty rows are common (more than one
   // per 256-entry chunk on average: a tile chunk would zero long runs of them, merge tiles count rows
-  // as work); else the tile kernel (nnz-balanced chunks) for skewed rows or nnz >= 2^20; else the
-  // stream kernel (warp per 32 rows), whose single launch is fastest on small regular matrices.
+  // as work); else the tile kernel (nnz-balanced chunks) for skewed rows or nnz >= 2^20 -- with row
+  // ids from a row-start bitmap when no row is empty (variant 4), from row_ptr otherwise (3); else
+  // the stream kernel (warp per 32 rows), whose single launch is fastest on small regular matrices.
   const long long avg = std::max(1LL, z / m);
   if (a.empty_rows * 256 > (long long)z) f->csr_variant = 1;
-  else if (mx > 4 * avg + 32 || z >= (1LL << 20)) f->csr_variant = 3;
+  else if (mx > 4 * avg + 32 || z >= (1LL << 20)) f->csr_variant = a.empty_rows == 0 ? 4 : 3;
   else f->csr_variant = 2;
-  if (o.csr_variant >= 0 && o.csr_variant <= 3) f->csr_variant = o.csr_variant;
+  if (o.csr_variant >= 0 && o.csr_variant <= 4) f->csr_variant = o.csr_variant;
 }
 
 static sfs_status check_csr(const sfs_csr* A) {
@@ -363,10 +364,12 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         A->work = own(csr_merge_work_bytes(m, z, d.dtype));
         if (!A->work) return bail(SFS_ERR_OOM, "csr merge carries");
         TRY_CUDA(launch_csr_merge_prepare((const int*)A->ptr[0], m, z, A->work, s));
-      } else if (A->variant == 3 && z > 0) {
-        A->work = own(csr_tile_work_bytes(m, z));
+      } else if ((A->variant == 3 || A->variant == 4) && z > 0) {
+        if (A->variant == 4 && f.nnz_min < 1) A->variant = 3;  // the row-start bitmap needs every row non-empty
+        const int bitmap = A->variant == 4;
+        A->work = own(csr_tile_work_bytes(m, z, bitmap));
         if (!A->work) return bail(SFS_ERR_OOM, "csr tile partition");
-        TRY_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, s));
+        TRY_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, bitmap, s));
       }
       break;
     }

@@ -98,8 +98,8 @@ int spmv_kernels_per_call(const Matrix* A);
 cudaError_t launch_spmv(const Matrix* A, const void* x, void* y, cudaStream_t s);
 size_t csr_merge_work_bytes(long long m, long long z, int dtype);
 cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s);
-size_t csr_tile_work_bytes(long long m, long long z);
-cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s);
+size_t csr_tile_work_bytes(long long m, long long z, int bitmap);
+cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s);
 int csr_vector_tpv(long long m, long long z);
 int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
@@ -125,7 +125,8 @@ struct Matrix {
   void* owned[8] = {nullptr};  // buffers to free
   int n_owned = 0;
   long long bytes = 0;
-  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile; HYB: 1 = one launch (ptr[5] = ovf)
+  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile, 4 tile + row-start bitmap;
+                               // HYB: 1 = one launch (ptr[5] = ovf)
   void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;
 };

@@ -462,12 +462,17 @@ __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, lo
   }
 }
 
-template <typename T, bool VEC>
+// BM (variant 4, matrices without empty rows): the row of every entry comes from a row-start bitmap
+// built with the handle (bit k set iff entry k starts a row, z/8 bytes): lane l's 8 entries are byte l
+// of the chunk's 32-byte bitmap, row = a - 1 + (row starts up to the entry), a warp scan of the bytes'
+// popcounts -- no row_ptr loads and no shared-memory marks on the chunk's critical path.
+template <typename T, bool VEC, bool BM = false>
 __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const int* __restrict__ col,
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
                                               const int* __restrict__ ca, int* __restrict__ carry_row,
-                                              acc_t* __restrict__ carry_val, int* head) {
+                                              acc_t* __restrict__ carry_val, int* head,
+                                              const unsigned* __restrict__ bm = nullptr) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
   const long long cb = warp * cpw;
@@ -481,10 +486,13 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     if (row < own_lo) { out_row = row; out_val = v; }
     else y[row] = (T)v;
   };
+  int a_run = own_lo;  // BM: first row starting at or after the chunk start
   for (long long ch = cb; ch < ce; ch++) {
     const long long k0 = ch * kTChunk;
     const long long k = k0 + l * kTV;
-    const int a_lo = __ldg(ca + ch), a_hi = __ldg(ca + ch + 1);
+    const int a_lo = BM ? 0 : __ldg(ca + ch), a_hi = BM ? 0 : __ldg(ca + ch + 1);
+    unsigned sb = 0;
+    if (BM) sb = (__ldg(bm + ch * (kTChunk / 32) + (l >> 2)) >> ((l & 3) * 8)) & 0xFFu;
     acc_t p[kTV];
     {
       int c[kTV];
@@ -503,6 +511,20 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
 #pragma unroll
       for (int i = 0; i < kTV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
     }
+    int r[kTV];
+    if (BM) {
+      const int cnt = __popc(sb);
+      int inc = cnt;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const int u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (l >= o) inc += u;
+      }
+      const int base = a_run - 1 + inc - cnt;
+#pragma unroll
+      for (int i = 0; i < kTV; i++) r[i] = base + __popc(sb & ((2u << i) - 1u));
+      a_run += __shfl_sync(0xffffffffu, inc, 31);
+    } else {
     // start marks of the rows beginning in this chunk (non-empty rows start at distinct positions)
     reinterpret_cast<int4*>(head)[2 * l] = make_int4(-1, -1, -1, -1);
     reinterpret_cast<int4*>(head)[2 * l + 1] = make_int4(-1, -1, -1, -1);
@@ -513,7 +535,6 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
       else y[r] = T(0);
     }
     __syncwarp();
-    int r[kTV];
     {
       const int4 h0 = reinterpret_cast<const int4*>(head)[2 * l], h1 = reinterpret_cast<const int4*>(head)[2 * l + 1];
       const int hv[kTV] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w};
@@ -535,6 +556,7 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
       for (int i = 0; i < kTV; i++) r[i] = r[i] > ex ? r[i] : ex;
     }
     __syncwarp();  // head is rewritten by the next chunk
+    }
     // segmented reduction of (r[i], p[i]) exactly as in the COO kernel; padding items (past z) have
     // p = 0 and the last row
     const int rf = r[0], rl = r[kTV - 1];
@@ -590,19 +612,29 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
 }
 
 // blockDim is 64, 128 or 256 (smaller CTAs spread a small matrix's few warps over more SMs)
-template <typename T, bool VEC>
+template <typename T, bool VEC, bool BM>
 __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
                                                                const int* __restrict__ ca, int* __restrict__ carry_row,
-                                                               acc_t* __restrict__ carry_val) {
-  __shared__ __align__(16) int s_head[kTThreads / 32][kTChunk];
+                                                               acc_t* __restrict__ carry_val,
+                                                               const unsigned* __restrict__ bm) {
+  __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
   pdl_wait();
   pdl_trigger();  // the fixup kernel launches now and waits for this grid to finish
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (warp < nwarps)
-    csr_tile_warp<T, VEC>(rp, col, val, x, y, m, z, cpw, warp, ca, carry_row, carry_val, s_head[threadIdx.x >> 5]);
+    csr_tile_warp<T, VEC, BM>(rp, col, val, x, y, m, z, cpw, warp, ca, carry_row, carry_val,
+                              s_head[BM ? 0 : threadIdx.x >> 5], bm);
+}
+
+// row-start bitmap of a CSR without empty rows: bit k set iff entry k is the first of its row
+__global__ void k_row_starts(const int* __restrict__ rp, long long m, unsigned* __restrict__ bm) {
+  for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (long long)gridDim.x * blockDim.x) {
+    const int k = __ldg(rp + r);
+    atomicOr(bm + (k >> 5), 1u << (k & 31));
+  }
 }
 
 // ======================================================================== COO (also the COO part of HYB)
@@ -963,6 +995,7 @@ struct TileWork {
   int* a;
   int* crow;
   acc_t* cval;
+  unsigned* bm;  // variant 4: row-start bitmap, nchunks * 8 words
 };
 TileWork tile_work(void* base, const TileGeom& g) {
   TileWork w;
@@ -972,6 +1005,8 @@ TileWork tile_work(void* base, const TileGeom& g) {
   w.crow = (int*)p;
   p += al256(sizeof(int) * g.nwarps);
   w.cval = (acc_t*)p;
+  p += al256(sizeof(acc_t) * g.nwarps);
+  w.bm = (unsigned*)p;
   return w;
 }
 
@@ -1013,7 +1048,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       const int* rp = (const int*)A->ptr[0];
       const int* col = (const int*)A->ptr[1];
       const T* val = (const T*)A->ptr[2];
-      if (A->variant == 3) {
+      if (A->variant == 3 || A->variant == 4) {
         if (z == 0) {
           e = launch_zero<T>(y, m, s);
           break;
@@ -1028,9 +1063,10 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const bool vec = ((((uintptr_t)col) | ((uintptr_t)val)) % 32) == 0;
         auto go = [&](auto kern) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a, w.crow,
-                          w.cval);
+                          w.cval, (const unsigned*)w.bm);
         };
-        e = vec ? go(k_spmv_csr_tile<T, true>) : go(k_spmv_csr_tile<T, false>);
+        if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>) : go(k_spmv_csr_tile<T, false, true>);
+        else e = vec ? go(k_spmv_csr_tile<T, true, false>) : go(k_spmv_csr_tile<T, false, false>);
         if (e == cudaSuccess)
           e = launch_k(k_spmv_csr_merge_fixup<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, (const int*)w.crow,
                        (const acc_t*)w.cval, g.nwarps, m, y);
@@ -1141,17 +1177,25 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
   return cudaGetLastError();
 }
 
-size_t csr_tile_work_bytes(long long m, long long z) {
+size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
   (void)m;
   const TileGeom g = tile_geom(z);
-  return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) + al256(sizeof(acc_t) * g.nwarps);
+  return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) + al256(sizeof(acc_t) * g.nwarps) +
+         (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0);
 }
 
-cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s) {
+cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
   const TileGeom g = tile_geom(z);
   TileWork w = tile_work(work, g);
   k_csr_tile_partition<<<grid_cap(g.nchunks + 1, 256, 8), 256, 0, s>>>(rp, m, g.nchunks, w.a);
   count_launch();
+  if (bitmap) {
+    cudaError_t e = cudaMemsetAsync(w.bm, 0, sizeof(unsigned) * g.nchunks * (kTChunk / 32), s);
+    count_launch();
+    if (e != cudaSuccess) return e;
+    k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm);
+    count_launch();
+  }
   return cudaGetLastError();
 }
 
@@ -1174,7 +1218,7 @@ int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) 
 
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
-    case SFS_CSR: return (A->variant == 1 || (A->variant == 3 && A->nnz > 0)) ? 2 : 1;
+    case SFS_CSR: return (A->variant == 1 || ((A->variant == 3 || A->variant == 4) && A->nnz > 0)) ? 2 : 1;
     case SFS_COO: return A->nnz > 0 ? 2 : 1;
     case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? 2 : 1;
     default: return 1;

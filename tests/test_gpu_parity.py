@@ -75,7 +75,7 @@ def test_conversions_bit_exact(name):
 
 
 @pytest.mark.parametrize("name", NAMES)
-@pytest.mark.parametrize("variant", [0, 1, 2, 3])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
 def test_spmv_tolerance(name, variant):
     A = cases()[name]
     fo = oracle.features(A.m, A.n, A.rp, A.col)
@@ -233,7 +233,7 @@ def test_launch_count_increases():
     assert sfs.launch_count() - c0 == 6  # zero kernel + COO kernel per COO SpMV
 
 
-def _tile_edge_csr(dtype, cap=None):
+def _tile_edge_csr(dtype, cap=None, no_empty=False):
     """Rows that stress the CSR tile kernel (variant 3): leading / trailing / mid-matrix runs of empty
     rows, rows of exactly 255/256/257/512 entries, one row of 400,000 entries spanning many warp
     ranges, and nnz large enough (> 148*4*8 chunks of 256) that each warp owns several chunks.
@@ -250,6 +250,8 @@ def _tile_edge_csr(dtype, cap=None):
     if cap is not None:
         lens = np.minimum(lens, cap)
         lens[rng.integers(0, m, 3000)] = cap  # many rows of exactly one chunk
+    if no_empty:
+        lens = np.maximum(lens, 1)
     rp = np.zeros(m + 1, np.int64)
     np.cumsum(lens, out=rp[1:])
     z = int(rp[-1])
@@ -328,3 +330,22 @@ def test_split_rows_and_gaps(shape):
         M = sfs.convert(dA, fmt, opts)
         check_spmv(A, fmt, M, x, A.dtype, ctx=f"{shape}/{sfs.FORMAT_NAMES[fmt]}")
         M.free()
+
+
+@pytest.mark.parametrize("cap", [None, 256])
+@pytest.mark.parametrize("dtype", [sfsgen.F64, sfsgen.F32])
+def test_csr_bitmap_tile(dtype, cap):
+    """CSR variant 4 (tile kernel with row ids from a row-start bitmap) on rows of 1..400,000 entries,
+    rows of exactly 255/256/257/512, a row spanning many warp ranges; with empty rows present the
+    handle falls back to the row_ptr tile kernel (variant 3)."""
+    A = _tile_edge_csr(dtype, cap, no_empty=True)
+    x = sfsgen.vector(6, A.n, A.dtype)
+    M = sfs.convert(to_dev(A), sfs.CSR, sfs.default_opts(csr_variant=4))
+    assert M.layout().variant == 4
+    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="bitmap-tile")
+    M.free()
+    B = _tile_edge_csr(dtype, cap)
+    M = sfs.convert(to_dev(B), sfs.CSR, sfs.default_opts(csr_variant=4))
+    assert M.layout().variant == 3
+    check_spmv(B, sfs.CSR, M, x[:B.n] if len(x) >= B.n else sfsgen.vector(6, B.n, B.dtype), B.dtype, ctx="bitmap-fallback")
+    M.free()

@@ -26,6 +26,7 @@ def hyb_rowwise(f, z):
 def kernels_of(fmt, f, z):
     if fmt == 0:
         return {2: ["k_spmv_csr_stream"], 3: ["k_spmv_csr_tile", "k_spmv_csr_merge_fixup"],
+                4: ["k_spmv_csr_tile", "k_spmv_csr_merge_fixup"],
                 1: ["k_spmv_csr_merge", "k_spmv_csr_merge_fixup"], 0: ["k_spmv_csr_vector"]}[f["csr_variant"]]
     if fmt == 1:
         return ["k_zero", "k_spmv_coo"]
