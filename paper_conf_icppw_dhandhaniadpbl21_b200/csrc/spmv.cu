@@ -423,9 +423,11 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
 // the rows that START in chunk c are [a_c, a_{c+1}), a_c = lower_bound(rp[0..m), 256 c) (computed
 // once per matrix); each non-empty one marks its start position, a max-scan carries the marks to
 // every entry, seeded with a_c - 1 (the row open at the chunk start).  Empty rows are zeroed by the
-// chunk that owns them.  Rows starting inside the warp's range are finished with plain stores; the
-// one row open at the range start goes to a per-warp carry that the fixup kernel adds (atomically,
-// after this grid completes).  No zero pass, no row array: CSR's own bytes only.
+// chunk that owns them.  Rows lying inside one warp's range are finished with plain stores; a row
+// split across ranges (one per range boundary, listed per matrix) is zeroed by k_zero_rows ahead of
+// this grid and gets every piece by atomicAdd.  k_zero_rows releases this kernel at once (PDL), so
+// the first chunk's loads and x gathers overlap it; the kernel waits before touching y.  No full zero
+// pass, no row array: CSR's own bytes only.
 constexpr int kTThreads = 256;
 constexpr int kTV = 8;
 constexpr int kTChunk = 32 * kTV;
@@ -470,20 +472,21 @@ template <typename T, bool VEC, bool BM = false>
 __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const int* __restrict__ col,
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
-                                              const int* __restrict__ ca, int* __restrict__ carry_row,
-                                              acc_t* __restrict__ carry_val, int* head,
-                                              const unsigned* __restrict__ bm = nullptr) {
+                                              const int* __restrict__ ca, const int* __restrict__ srow,
+                                              long long nwarps, int* head, const unsigned* __restrict__ bm = nullptr) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
   const long long cb = warp * cpw;
   const long long ce = cb + cpw < nchunks ? cb + cpw : nchunks;
   const int own_lo = __ldg(ca + cb);  // rows >= own_lo start inside this range
+  // the row split at the boundary with the next range (m: none); srow[w] rows were zeroed by
+  // k_zero_rows before this grid touched y, and every piece of them is added atomically
+  const int next_split = warp + 1 < nwarps ? __ldg(srow + warp + 1) : (int)m;
   int open_row = -1;                  // row left open at the previous chunk's end (all lanes agree)
   acc_t open = 0;
-  int out_row = (int)m;               // the row open at the range start, for the fixup
-  acc_t out_val = 0;
+  bool waited = false;                // PDL: loads of the first chunk overlap k_zero_rows
   auto emit = [&](int row, acc_t v) {
-    if (row < own_lo) { out_row = row; out_val = v; }
+    if (row < own_lo) atomicAdd(y + row, (T)v);  // the piece of the row carried into this range
     else y[row] = (T)v;
   };
   int a_run = own_lo;  // BM: first row starting at or after the chunk start
@@ -510,6 +513,11 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
       }
 #pragma unroll
       for (int i = 0; i < kTV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
+    }
+    if (!waited) {
+      pdl_wait();
+      pdl_trigger();
+      waited = true;
     }
     int r[kTV];
     if (BM) {
@@ -602,12 +610,9 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     open_row = __shfl_sync(0xffffffffu, rl, 31);
     open = __shfl_sync(0xffffffffu, S, 31);
   }
-  if (l == 0 && open_row >= 0) emit(open_row, open);  // a partial if the row continues past the range
-  const unsigned has = __ballot_sync(0xffffffffu, out_row < m);
-  if (has) {
-    if (l == __ffs(has) - 1) { carry_row[warp] = out_row; carry_val[warp] = out_val; }
-  } else if (l == 0) {
-    carry_row[warp] = (int)m;
+  if (l == 0 && open_row >= 0) {  // a piece of a split row if it continues past the range
+    if (open_row == next_split) atomicAdd(y + open_row, (T)open);
+    else emit(open_row, open);
   }
 }
 
@@ -617,16 +622,44 @@ __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __res
                                                                const T* __restrict__ val, const T* __restrict__ x,
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
-                                                               const int* __restrict__ ca, int* __restrict__ carry_row,
-                                                               acc_t* __restrict__ carry_val,
+                                                               const int* __restrict__ ca, const int* __restrict__ srow,
                                                                const unsigned* __restrict__ bm) {
   __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
-  pdl_wait();
-  pdl_trigger();  // the fixup kernel launches now and waits for this grid to finish
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (warp < nwarps)
-    csr_tile_warp<T, VEC, BM>(rp, col, val, x, y, m, z, cpw, warp, ca, carry_row, carry_val,
-                              s_head[BM ? 0 : threadIdx.x >> 5], bm);
+    csr_tile_warp<T, VEC, BM>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps, s_head[BM ? 0 : threadIdx.x >> 5],
+                              bm);
+  else
+    pdl_wait();
+  pdl_trigger();
+}
+
+// Rows split across two warp ranges of the tile kernel (one per range boundary, precomputed): zeroed
+// ahead of the tile grid, which adds their pieces atomically.  Releases the tile kernel at once so
+// that its first loads overlap this kernel (the tile kernel waits before touching y).
+template <typename T>
+__global__ void k_zero_rows(T* __restrict__ y, const int* __restrict__ srow, long long n, long long m) {
+  pdl_wait();
+  pdl_trigger();
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (long long)gridDim.x * blockDim.x) {
+    const int r = srow[i];
+    if (r < m) y[r] = T(0);
+  }
+}
+
+// srow[w] = the row holding the first entry of warp w's range if it started before it, else m
+__global__ void k_tile_split_rows(const int* __restrict__ rp, long long m, long long cpw, long long nwarps,
+                                  int* __restrict__ srow) {
+  for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nwarps; w += (long long)gridDim.x * blockDim.x) {
+    const long long kb = w * cpw * kTChunk;
+    long long lo = 0, hi = m;  // last row r with rp[r] <= kb
+    while (lo < hi) {
+      const long long mid = (lo + hi + 1) >> 1;
+      if (rp[mid] <= kb) lo = mid;
+      else hi = mid - 1;
+    }
+    srow[w] = (w > 0 && rp[lo] < kb) ? (int)lo : (int)m;
+  }
 }
 
 // row-start bitmap of a CSR without empty rows: bit k set iff entry k is the first of its row
@@ -992,9 +1025,8 @@ MergeWork merge_work(void* base, long long tiles) {
 }
 
 struct TileWork {
-  int* a;
-  int* crow;
-  acc_t* cval;
+  int* a;        // a_c = lower_bound(rp, 256 c), c = 0..nchunks
+  int* srow;     // row split at the start of each warp range (m: none)
   unsigned* bm;  // variant 4: row-start bitmap, nchunks * 8 words
 };
 TileWork tile_work(void* base, const TileGeom& g) {
@@ -1002,10 +1034,8 @@ TileWork tile_work(void* base, const TileGeom& g) {
   char* p = (char*)base;
   w.a = (int*)p;
   p += al256(sizeof(int) * (g.nchunks + 1));
-  w.crow = (int*)p;
+  w.srow = (int*)p;
   p += al256(sizeof(int) * g.nwarps);
-  w.cval = (acc_t*)p;
-  p += al256(sizeof(acc_t) * g.nwarps);
   w.bm = (unsigned*)p;
   return w;
 }
@@ -1062,14 +1092,14 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         // borrowed arrays (e.g. a row block of a larger CSR) may not be 32 B aligned: scalar loads
         const bool vec = ((((uintptr_t)col) | ((uintptr_t)val)) % 32) == 0;
         auto go = [&](auto kern) {
-          return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a, w.crow,
-                          w.cval, (const unsigned*)w.bm);
+          return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
+                          (const int*)w.srow, (const unsigned*)w.bm);
         };
-        if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>) : go(k_spmv_csr_tile<T, false, true>);
-        else e = vec ? go(k_spmv_csr_tile<T, true, false>) : go(k_spmv_csr_tile<T, false, false>);
-        if (e == cudaSuccess)
-          e = launch_k(k_spmv_csr_merge_fixup<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, (const int*)w.crow,
-                       (const acc_t*)w.cval, g.nwarps, m, y);
+        e = launch_k(k_zero_rows<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, y, (const int*)w.srow, g.nwarps, m);
+        if (e == cudaSuccess) {
+          if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>) : go(k_spmv_csr_tile<T, false, true>);
+          else e = vec ? go(k_spmv_csr_tile<T, true, false>) : go(k_spmv_csr_tile<T, false, false>);
+        }
       } else if (A->variant == 2) {
         const long long groups = ceil_div(m, 32);
         const long long windows = ceil_div(z, 32 * stream_u<T>());  // ~ windows over all groups
@@ -1180,7 +1210,7 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
   (void)m;
   const TileGeom g = tile_geom(z);
-  return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) + al256(sizeof(acc_t) * g.nwarps) +
+  return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) +
          (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0);
 }
 
@@ -1188,6 +1218,8 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
   const TileGeom g = tile_geom(z);
   TileWork w = tile_work(work, g);
   k_csr_tile_partition<<<grid_cap(g.nchunks + 1, 256, 8), 256, 0, s>>>(rp, m, g.nchunks, w.a);
+  count_launch();
+  k_tile_split_rows<<<grid_cap(g.nwarps, 256, 8), 256, 0, s>>>(rp, m, g.cpw, g.nwarps, w.srow);
   count_launch();
   if (bitmap) {
     cudaError_t e = cudaMemsetAsync(w.bm, 0, sizeof(unsigned) * g.nchunks * (kTChunk / 32), s);
