@@ -640,7 +640,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   std::vector<DevCSR> d(n);
   std::vector<FeatWork> w(n);
   std::vector<sfs_status> mst(n, SFS_OK);
-  std::vector<cudaEvent_t> fe0(n, nullptr), fe1(n, nullptr);
+  std::vector<cudaEvent_t> fe0(n, nullptr), fe1(n, nullptr), ce(n, nullptr);
   DevAggr* ha = nullptr;
   TRY_CUDA(cudaMallocHost(&ha, sizeof(DevAggr) * std::max<int64_t>(n, 1)));
   for (int64_t i = 0; i < n; i++) {
@@ -655,42 +655,45 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
       TRY_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
       break;
     }
-  // ---- phase 1: stage + features of every matrix, one synchronisation
-  for (int64_t i = 0; i < n; i++) {
-    sfs_status st = check_csr(&mats[i]);
-    // host inputs: stage on the copy stream so the H2D of matrix i+1 overlaps the features of i
-    if (st == SFS_OK) st = stage(&mats[i], d[i], cs ? cs : s, true);
-    if (st == SFS_OK && d[i].host && cs) {
-      cudaEvent_t ec = ev.get();
-      cudaEventRecord(ec, cs);
-      cudaStreamWaitEvent(s, ec, 0);
+  // Chunks.  A device-resident corpus is one chunk: every feature pass, one synchronisation (the host
+  // needs the features to enqueue the race), then the whole race enqueued.  Host-memory inputs come in
+  // chunks of 1, 2, 4, ... matrices: the H2D copies of chunk c+1 (copy stream) run during the race of
+  // chunk c, so only the first matrix's copy is exposed.  The copies are ~10x faster than the race
+  // consumes the same bytes, so each chunk's inputs are resident before its predecessor's race ends.
+  std::vector<int64_t> cb{0};
+  if (cs) {
+    for (int64_t len = 1; cb.back() < n; len *= 2) cb.push_back(std::min<int64_t>(n, cb.back() + len));
+  } else if (n > 0) {
+    cb.push_back(n);
+  }
+  const int nchunks = (int)cb.size() - 1;
+  // stage: (host inputs) allocate + H2D on the copy stream, one event per matrix
+  auto stage_chunk = [&](int c) {
+    for (int64_t i = cb[c]; i < cb[c + 1]; i++) {
+      sfs_status st = check_csr(&mats[i]);
+      if (st == SFS_OK) st = stage(&mats[i], d[i], cs ? cs : s, true);
+      if (st == SFS_OK && d[i].host && cs) {
+        ce[i] = ev.get();
+        cudaEventRecord(ce[i], cs);
+      }
+      mst[i] = st;
     }
-    if (st == SFS_OK) {
+  };
+  // features on the compute stream (after the matrix's copy)
+  auto features_chunk = [&](int c) {
+    for (int64_t i = cb[c]; i < cb[c + 1]; i++) {
+      if (mst[i] != SFS_OK) continue;
+      if (ce[i]) cudaStreamWaitEvent(s, ce[i], 0);
       fe0[i] = ev.get();
       fe1[i] = ev.get();
       cudaEventRecord(fe0[i], s);
-      st = features_device(d[i], o, w[i], &ha[i], s);
+      mst[i] = features_device(d[i], o, w[i], &ha[i], s);
       cudaEventRecord(fe1[i], s);
     }
-    mst[i] = st;
-  }
-  cudaError_t e = cudaStreamSynchronize(s);
-  if (e != cudaSuccess) {
-    cudaFreeHost(ha);
-    cudaStreamDestroy(cap);
-    if (up) cudaStreamDestroy(up);
-    if (cs) cudaStreamDestroy(cs);
-    return cuda_fail(e, "feature phase");
-  }
-  for (int64_t i = 0; i < n; i++) {
-    if (mst[i] == SFS_OK) mst[i] = features_finish(d[i], o, ha[i], &feats[i], s);
-    if (mst[i] == SFS_OK) labels[i].t_features_us = elapsed_us(fe0[i], fe1[i]);
-  }
-  // ---- phase 2: the race; everything enqueued, no host synchronisation
+  };
   using clk = std::chrono::steady_clock;
   const bool prof = getenv("SFS_PROFILE") != nullptr;
-  double t_graph = 0, t_inst = 0, t_conv = 0, t_warm = 0;
-  const auto t_phase2 = clk::now();
+  double t_graph = 0, t_inst = 0, t_conv = 0, t_warm = 0, t_sync = 0;
   struct Timed {
     int64_t i;
     int f;
@@ -702,18 +705,27 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   std::vector<cudaGraph_t> graphs;
   void* flush = nullptr;
   size_t flush_bytes = 0;
-  if (o.cold) {
+  auto cleanup = [&]() {
+    for (auto ge : execs) cudaGraphExecDestroy(ge);
+    for (auto g : graphs) cudaGraphDestroy(g);
+    cudaStreamDestroy(cap);
+    if (up) cudaStreamDestroy(up);
+    if (cs) cudaStreamDestroy(cs);
+    cudaFreeHost(ha);
+  };
+  if (o.cold && n > 0) {
     int dev = 0, l2 = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
     flush_bytes = (size_t)std::max(l2, 1 << 20) * 2;
     flush = dalloc(flush_bytes, s);
   }
-  for (int64_t i = 0; i < n; i++) {
+  // the race of one matrix: every admissible format converted, warmed up and timed; nothing synchronises
+  auto race_one = [&](int64_t i) {
     sfs_label_t& L = labels[i];
     if (mst[i] != SFS_OK) {
       L.matrix_status = mst[i];
-      continue;
+      return;
     }
     const sfs_features_t& F = feats[i];
     L.admissible_mask = F.admissible_mask;
@@ -732,7 +744,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
       L.matrix_status = SFS_ERR_OOM;
       dfree(y, s);
       dfree(xo, s);
-      continue;
+      return;
     }
     for (int f = 0; f < SFS_NFMT; f++) {
       L.bytes[f] = sfs_spmv_bytes(&F, (sfs_format)f, (sfs_dtype)D.dtype);
@@ -813,11 +825,34 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     }
     dfree(y, s);
     dfree(xo, s);
+  };
+  const auto t_phase2 = clk::now();
+  if (nchunks > 0) {
+    stage_chunk(0);
+    features_chunk(0);
   }
-  // release the per-matrix feature workspaces and staged inputs (stream-ordered)
-  for (int64_t i = 0; i < n; i++) {
-    dfree(w[i].base, s);
-    unstage(d[i], s);
+  cudaError_t e = cudaSuccess;
+  for (int c = 0; c < nchunks; c++) {
+    const auto ts0 = clk::now();
+    e = cudaStreamSynchronize(s);  // this chunk's features (and the previous chunk's race) are done
+    t_sync += std::chrono::duration<double>(clk::now() - ts0).count();
+    if (e != cudaSuccess) {
+      cleanup();
+      return cuda_fail(e, c == 0 ? "feature phase" : "race");
+    }
+    for (int64_t i = cb[c]; i < cb[c + 1]; i++) {
+      if (mst[i] == SFS_OK) mst[i] = features_finish(d[i], o, ha[i], &feats[i], s);
+      if (mst[i] == SFS_OK) labels[i].t_features_us = elapsed_us(fe0[i], fe1[i]);
+    }
+    if (c + 1 < nchunks) stage_chunk(c + 1);  // H2D of the next chunk overlaps this chunk's race
+    for (int64_t i = cb[c]; i < cb[c + 1]; i++) race_one(i);
+    // release the chunk's feature workspaces and staged inputs (stream-ordered)
+    for (int64_t i = cb[c]; i < cb[c + 1]; i++) {
+      dfree(w[i].base, s);
+      w[i].base = nullptr;
+      unstage(d[i], s);
+    }
+    if (c + 1 < nchunks) features_chunk(c + 1);
   }
   if (flush) dfree(flush, s);
   const auto t_enq = clk::now();
@@ -825,17 +860,13 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   if (prof) {
     const auto t_end = clk::now();
     fprintf(stderr,
-            "[sfs] label_corpus n=%lld: enqueue %.1f ms (convert %.1f, warmup %.1f, graph capture %.1f + instantiate "
-            "%.1f ms), sync wait %.1f ms\n",
-            (long long)n, 1e3 * std::chrono::duration<double>(t_enq - t_phase2).count(), 1e3 * t_conv, 1e3 * t_warm,
-            1e3 * (t_graph - t_inst), 1e3 * t_inst, 1e3 * std::chrono::duration<double>(t_end - t_enq).count());
+            "[sfs] label_corpus n=%lld chunks=%d: enqueue %.1f ms (convert %.1f, warmup %.1f, graph capture %.1f + "
+            "instantiate %.1f ms, chunk syncs %.1f ms), sync wait %.1f ms\n",
+            (long long)n, nchunks, 1e3 * std::chrono::duration<double>(t_enq - t_phase2).count(), 1e3 * t_conv,
+            1e3 * t_warm, 1e3 * (t_graph - t_inst), 1e3 * t_inst, 1e3 * t_sync,
+            1e3 * std::chrono::duration<double>(t_end - t_enq).count());
   }
-  for (auto ge : execs) cudaGraphExecDestroy(ge);
-  for (auto g : graphs) cudaGraphDestroy(g);
-  cudaStreamDestroy(cap);
-  if (up) cudaStreamDestroy(up);
-  if (cs) cudaStreamDestroy(cs);
-  cudaFreeHost(ha);
+  cleanup();
   if (e != cudaSuccess) return cuda_fail(e, "race");
   for (auto& T : timed) {
     sfs_label_t& L = labels[T.i];

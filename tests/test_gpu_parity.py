@@ -221,6 +221,33 @@ def test_label_corpus_invalid_matrix_does_not_abort():
     assert labs[1]["matrix_status"] == 0 and labs[1]["label"] >= 0
 
 
+def test_label_corpus_host_inputs_chunked():
+    """Host-memory corpus: inputs staged in chunks of 1, 2, 4, ... matrices, each chunk's H2D overlapping the
+    previous chunk's race.  Features bit-exact, statuses per matrix (an invalid one in the middle of a chunk),
+    the same admissible formats raced as from device memory."""
+    import torch
+    names = ["laplace64", "band", "blockdiag32", "uniform", "powerlaw32", "rmat14", "empty", "tiny4x4"]
+    A = {k: cases()[k] for k in names}
+    bad = sfsgen.CSR(A["band"].m, A["band"].n, A["band"].rp.copy(), A["band"].col.copy(), A["band"].val)
+    bad.col[5] = bad.col[4]
+    order = names[:4] + ["bad"] + names[4:]
+    A["bad"] = bad
+    pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
+    mats = [sfs.Csr(A[k].m, A[k].n, pin(A[k].rp), pin(A[k].col), pin(A[k].val),
+                    pin(sfsgen.vector(3, A[k].n, A[k].dtype))) for k in order]
+    feats, labs = sfs.label_corpus(mats, sfs.default_opts(reps=5, warmup=1))
+    for k, f, L in zip(order, feats, labs):
+        if k == "bad":
+            assert L["matrix_status"] == sfs.ERR_INVALID_CSR and L["label"] == -1
+            continue
+        fo = oracle.features(A[k].m, A[k].n, A[k].rp, A[k].col)
+        assert_features_equal(f, fo, k)
+        assert L["matrix_status"] == 0
+        ran = [i for i in range(5) if L["status"][i] == 0]
+        assert ran == [i for i in range(5) if (fo["admissible_mask"] >> i) & 1], k
+        assert L["label"] == oracle.label(np.array(L["t_spmv_us"], np.float64), sum(1 << i for i in ran))
+
+
 def test_launch_count_increases():
     import torch
     A = cases()["band"]

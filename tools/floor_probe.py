@@ -11,3 +11,7 @@ for pdl in ["1"]:
     feats, labs = sfs.label_corpus(mats, sfs.default_opts())
     for M, L in zip(mats, labs):
         print(M.m, M.nnz, [round(v, 2) for v in L["t_spmv_us"]], L["csr_variant"])
+print("graphs:")
+feats, labs = sfs.label_corpus(mats, sfs.default_opts(use_graphs=1))
+for M, L in zip(mats, labs):
+    print(M.m, M.nnz, [round(v, 2) for v in L["t_spmv_us"]], L["csr_variant"])
