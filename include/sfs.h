@@ -162,6 +162,55 @@ sfs_status sfs_label_corpus(const sfs_csr *mats, int64_t n, const sfs_race_opts 
    dtype, n < 0 or a null pointer with n > 0. */
 sfs_status sfs_gather(sfs_dtype dtype, const void *src, const int32_t *idx, int64_t n, void *dst, void *stream);
 
+/* Row-partitioned SpMV with the halo exchange fused in (SURVEY §8(e) 2, §8(f) f3 "stores of y into
+   every peer's x"; y = A·x of P:L31 split by rows).  Rank k holds a row block of A with its columns
+   renumbered into x_ext = [ghosts below | own slice | ghosts above] and writes y into the own slice of
+   its next x_ext.  Each neighbour j needs some of those y entries as its ghosts; they form contiguous
+   runs of local rows (a banded/stencil block: one run per neighbour) and land in contiguous runs of
+   j's next x_ext.  sfs_spmv_push computes y = A·x and stores every y[r] with r in a run also into the
+   run's destination -- peer memory mapped into this process (NVLink P2P / symmetric memory, or plain
+   device memory when P ranks are simulated on one GPU) -- from the same kernel that computes it, so
+   the transfer overlaps the SpMV tile by tile.  Completion protocol (flags are uint32 in device
+   memory, monotonically increasing epochs):
+     start: every CTA waits until *wait_flag[i] >= wait_value for all i < nwait (acquire, system
+            scope) before reading x: the neighbours have pushed this epoch's ghosts into x and have
+            finished reading the buffer this call pushes into (double-buffered x_ext);
+     end:   after all CTAs' stores, the last CTA (counted in *counter, which it resets to 0) stores
+            sig_value into every *sig_flag[i] (release, system scope).
+   Fused in one kernel for DIA, ELL and the CSR stream kernel; the other kernels run as
+   wait kernel -> SpMV -> push kernel (same protocol, three launches).  Runs must not overlap and must
+   lie in [0, nrows).  INVALID_ARG for bad counts / null pointers, else as sfs_spmv.  Asynchronous. */
+#define SFS_MAX_PUSH 8
+#define SFS_MAX_PEERS 16
+typedef struct {
+  int32_t nseg;                              /* runs, <= SFS_MAX_PUSH */
+  int64_t seg_begin[SFS_MAX_PUSH];           /* local rows [seg_begin, seg_end) of y ... */
+  int64_t seg_end[SFS_MAX_PUSH];
+  void *seg_dst[SFS_MAX_PUSH];               /* ... also stored at seg_dst[r - seg_begin] (dtype) */
+  int32_t nwait;                             /* <= SFS_MAX_PEERS */
+  const uint32_t *wait_flag[SFS_MAX_PEERS];  /* this rank's flag slots, written by its neighbours */
+  uint32_t wait_value;
+  int32_t nsig;                              /* <= SFS_MAX_PEERS */
+  uint32_t *sig_flag[SFS_MAX_PEERS];         /* this rank's slot in each neighbour's flags */
+  uint32_t sig_value;
+  uint32_t *counter;                         /* device, zero before the first call; one per rank */
+} sfs_push_t;
+sfs_status sfs_spmv_push(sfs_format f, sfs_matrix A, const void *x, void *y, const sfs_push_t *push,
+                         void *stream);
+/* Peer memory for the push (plumbing; CUDA IPC): sfs_ipc_alloc allocates `bytes` of zeroed device memory
+   on the current device and writes its 64-byte IPC handle; another process on the node maps it with
+   sfs_ipc_open (peer access enabled lazily, so a buffer on another GPU is reached over NVLink) and
+   unmaps it with sfs_ipc_close; the owner frees it with sfs_ipc_free.  Synchronous; CUDA errors ->
+   SFS_ERR_CUDA. */
+sfs_status sfs_ipc_alloc(size_t bytes, void **ptr, uint8_t handle[64]);
+sfs_status sfs_ipc_open(const uint8_t handle[64], void **ptr);
+sfs_status sfs_ipc_close(void *ptr);
+sfs_status sfs_ipc_free(void *ptr);
+/* The push alone (no SpMV): stores src[r] (r in the runs) into the runs' destinations with the same
+   wait / signal protocol -- the initial ghost exchange before the first sfs_spmv_push.  src: nrows
+   entries of dtype (device).  One kernel launch. */
+sfs_status sfs_halo_push(sfs_dtype dtype, const void *src, int64_t nrows, const sfs_push_t *push, void *stream);
+
 sfs_status sfs_matrix_free(sfs_matrix A); /* stream-ordered on the stream it was created on */
 sfs_status sfs_matrix_describe(sfs_matrix A, sfs_layout_t *out);
 

@@ -95,6 +95,12 @@ def lib():
         L.sfs_convert.argtypes = [ctypes.POINTER(CsrStruct), _I32, ctypes.POINTER(RaceOpts), ctypes.POINTER(_P), _P]
         L.sfs_spmv.argtypes = [_I32, _P, _P, _P, _P]
         L.sfs_gather.argtypes = [_I32, _P, _P, _I64, _P, _P]
+        L.sfs_spmv_push.argtypes = [_I32, _P, _P, _P, ctypes.POINTER(PushStruct), _P]
+        L.sfs_halo_push.argtypes = [_I32, _P, _I64, ctypes.POINTER(PushStruct), _P]
+        L.sfs_ipc_alloc.argtypes = [ctypes.c_size_t, ctypes.POINTER(_P), ctypes.c_char_p]
+        L.sfs_ipc_open.argtypes = [ctypes.c_char_p, ctypes.POINTER(_P)]
+        L.sfs_ipc_close.argtypes = [_P]
+        L.sfs_ipc_free.argtypes = [_P]
         L.sfs_label_corpus.argtypes = [ctypes.POINTER(CsrStruct), _I64, ctypes.POINTER(RaceOpts),
                                        ctypes.POINTER(FeaturesStruct), ctypes.POINTER(LabelStruct), _P]
         L.sfs_matrix_free.argtypes = [_P]
@@ -247,6 +253,73 @@ def gather(src, idx, dst, stream=None):
     _check(lib().sfs_gather(dt, src.data_ptr(), idx.data_ptr(), idx.numel(), dst.data_ptr(), _stream_ptr(stream)),
            "sfs_gather")
     return dst
+
+
+MAX_PUSH = 8
+MAX_PEERS = 16
+
+
+class PushStruct(ctypes.Structure):
+    """sfs_push_t (include/sfs.h): runs of y rows also stored into peer memory, wait / signal flags."""
+    _fields_ = [("nseg", _I32), ("seg_begin", _I64 * MAX_PUSH), ("seg_end", _I64 * MAX_PUSH),
+                ("seg_dst", _P * MAX_PUSH), ("nwait", _I32), ("wait_flag", _P * MAX_PEERS), ("wait_value", _U32),
+                ("nsig", _I32), ("sig_flag", _P * MAX_PEERS), ("sig_value", _U32), ("counter", _P)]
+
+
+def push_struct(runs, wait_flags, wait_value, sig_flags, sig_value, counter) -> PushStruct:
+    """runs: [(begin, end, dst_address)]; flags / counter: device addresses (ints)."""
+    if len(runs) > MAX_PUSH or len(wait_flags) > MAX_PEERS or len(sig_flags) > MAX_PEERS:
+        raise SfsError(ERR_INVALID_ARG, "push plan too large")
+    p = PushStruct()
+    p.nseg = len(runs)
+    for i, (b, e, d) in enumerate(runs):
+        p.seg_begin[i], p.seg_end[i], p.seg_dst[i] = int(b), int(e), int(d)
+    p.nwait = len(wait_flags)
+    for i, f in enumerate(wait_flags):
+        p.wait_flag[i] = int(f)
+    p.wait_value = int(wait_value) & 0xFFFFFFFF
+    p.nsig = len(sig_flags)
+    for i, f in enumerate(sig_flags):
+        p.sig_flag[i] = int(f)
+    p.sig_value = int(sig_value) & 0xFFFFFFFF
+    p.counter = int(counter)
+    return p
+
+
+def spmv_push(fmt: int, A: Matrix, x, y, push: PushStruct, stream=None):
+    """y = A x with the halo push fused in (sfs_spmv_push); asynchronous on `stream`."""
+    _check(lib().sfs_spmv_push(fmt, A.handle, x.data_ptr(), y.data_ptr(), ctypes.byref(push), _stream_ptr(stream)),
+           "sfs_spmv_push")
+    return y
+
+
+def halo_push(src, push: PushStruct, stream=None):
+    """The push alone (sfs_halo_push): initial ghost exchange of a row-partitioned iteration."""
+    dt = F64 if src.element_size() == 8 else F32
+    _check(lib().sfs_halo_push(dt, src.data_ptr(), src.numel(), ctypes.byref(push), _stream_ptr(stream)),
+           "sfs_halo_push")
+
+
+def ipc_alloc(nbytes: int):
+    """Zeroed device memory shareable with other processes on the node: (address, 64-byte handle)."""
+    p, h = _P(), ctypes.create_string_buffer(64)
+    _check(lib().sfs_ipc_alloc(nbytes, ctypes.byref(p), h), "sfs_ipc_alloc")
+    return int(p.value), h.raw
+
+
+def ipc_open(handle: bytes) -> int:
+    """Map another process's ipc_alloc buffer (peer access over NVLink when it lives on another GPU)."""
+    p = _P()
+    _check(lib().sfs_ipc_open(ctypes.create_string_buffer(handle, 64), ctypes.byref(p)), "sfs_ipc_open")
+    return int(p.value)
+
+
+def ipc_close(addr: int):
+    _check(lib().sfs_ipc_close(addr), "sfs_ipc_close")
+
+
+def ipc_free(addr: int):
+    _check(lib().sfs_ipc_free(addr), "sfs_ipc_free")
 
 
 def label_corpus(mats: Sequence[Csr], opts: Optional[RaceOpts] = None, stream=None):

@@ -597,6 +597,75 @@ sfs_status sfs_gather(sfs_dtype dtype, const void* src, const int32_t* idx, int6
   return SFS_OK;
 }
 
+// Row-partitioned SpMV with the halo push fused in (include/sfs.h).
+static sfs_status check_push(const sfs_push_t* p, long long nrows) {
+  if (!p) return fail(SFS_ERR_INVALID_ARG, "null push plan");
+  if (p->nseg < 0 || p->nseg > SFS_MAX_PUSH || p->nwait < 0 || p->nwait > SFS_MAX_PEERS || p->nsig < 0 ||
+      p->nsig > SFS_MAX_PEERS)
+    return fail(SFS_ERR_INVALID_ARG, "push plan counts out of range");
+  if (!p->counter) return fail(SFS_ERR_INVALID_ARG, "push plan needs a counter");
+  for (int i = 0; i < p->nseg; i++) {
+    if (p->seg_begin[i] < 0 || p->seg_end[i] < p->seg_begin[i] || p->seg_end[i] > nrows || !p->seg_dst[i])
+      return fail(SFS_ERR_INVALID_ARG, "push run outside the row block or null destination");
+    for (int j = 0; j < i; j++)
+      if (p->seg_begin[i] < p->seg_end[j] && p->seg_begin[j] < p->seg_end[i])
+        return fail(SFS_ERR_INVALID_ARG, "push runs overlap");
+  }
+  for (int i = 0; i < p->nwait; i++)
+    if (!p->wait_flag[i]) return fail(SFS_ERR_INVALID_ARG, "null wait flag");
+  for (int i = 0; i < p->nsig; i++)
+    if (!p->sig_flag[i]) return fail(SFS_ERR_INVALID_ARG, "null signal flag");
+  return SFS_OK;
+}
+
+sfs_status sfs_spmv_push(sfs_format f, sfs_matrix Ah, const void* x, void* y, const sfs_push_t* push, void* stream) {
+  Matrix* A = (Matrix*)Ah;
+  if (!A || ((!x || !y) && A->m > 0)) return fail(SFS_ERR_INVALID_ARG, "null argument");
+  if ((int)f != A->fmt) return fail(SFS_ERR_INVALID_ARG, "format argument does not match the handle");
+  sfs_status st = check_push(push, A->m);
+  if (st != SFS_OK) return st;
+  TRY_CUDA(launch_spmv_push(A, x, y, *push, (cudaStream_t)stream));
+  return SFS_OK;
+}
+
+sfs_status sfs_halo_push(sfs_dtype dtype, const void* src, int64_t nrows, const sfs_push_t* push, void* stream) {
+  if ((dtype != SFS_F32 && dtype != SFS_F64) || nrows < 0 || (!src && nrows > 0))
+    return fail(SFS_ERR_INVALID_ARG, "bad dtype / source");
+  sfs_status st = check_push(push, nrows);
+  if (st != SFS_OK) return st;
+  TRY_CUDA(launch_halo_push(dtype, src, nrows, *push, (cudaStream_t)stream));
+  return SFS_OK;
+}
+
+sfs_status sfs_ipc_alloc(size_t bytes, void** ptr, uint8_t handle[64]) {
+  if (!ptr || !handle || bytes == 0) return fail(SFS_ERR_INVALID_ARG, "null argument / zero size");
+  static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
+  TRY_CUDA(cudaMalloc(ptr, bytes));
+  TRY_CUDA(cudaMemset(*ptr, 0, bytes));
+  cudaIpcMemHandle_t h;
+  TRY_CUDA(cudaIpcGetMemHandle(&h, *ptr));
+  memcpy(handle, &h, 64);
+  return SFS_OK;
+}
+
+sfs_status sfs_ipc_open(const uint8_t handle[64], void** ptr) {
+  if (!ptr || !handle) return fail(SFS_ERR_INVALID_ARG, "null argument");
+  cudaIpcMemHandle_t h;
+  memcpy(&h, handle, 64);
+  TRY_CUDA(cudaIpcOpenMemHandle(ptr, h, cudaIpcMemLazyEnablePeerAccess));
+  return SFS_OK;
+}
+
+sfs_status sfs_ipc_close(void* ptr) {
+  TRY_CUDA(cudaIpcCloseMemHandle(ptr));
+  return SFS_OK;
+}
+
+sfs_status sfs_ipc_free(void* ptr) {
+  TRY_CUDA(cudaFree(ptr));
+  return SFS_OK;
+}
+
 sfs_status sfs_matrix_free(sfs_matrix A) {
   matrix_free((Matrix*)A);
   return SFS_OK;

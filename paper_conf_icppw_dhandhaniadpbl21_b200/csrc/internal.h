@@ -106,6 +106,9 @@ cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t 
 // dst[i] = src[idx[i]], i < n (exchange.cu: halo send buffers of the row-partitioned SpMV)
 cudaError_t launch_gather(int dtype, const void* src, const int* idx, long long n, void* dst, cudaStream_t s);
 cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s);
+// fused SpMV + halo push (sfs_spmv_push) and the push alone (sfs_halo_push); `p` validated by the caller
+cudaError_t launch_spmv_push(const Matrix* A, const void* x, void* y, const sfs_push_t& p, cudaStream_t s);
+cudaError_t launch_halo_push(int dtype, const void* src, long long nrows, const sfs_push_t& p, cudaStream_t s);
 
 // ---------------------------------------------------------------- semi-supervised predictor (cluster.cu)
 struct ClusterModel;

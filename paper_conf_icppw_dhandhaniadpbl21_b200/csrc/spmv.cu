@@ -30,6 +30,8 @@
 #include <stdio.h>
 #include <stdlib.h>
 
+#include <algorithm>
+
 #include "common.cuh"
 #include "internal.h"
 
@@ -104,6 +106,137 @@ __global__ void k_zero(T* __restrict__ y, long long m) {
     y[i] = T(0);
 }
 
+// ======================================================================== fused halo push
+// sfs_spmv_push (include/sfs.h): the row-owning kernels (DIA, ELL, CSR stream) store each y[r] that a
+// neighbour needs as a ghost also into the neighbour's x_ext (peer memory), in the same instruction
+// stream that computes it.  PushParam<false> is empty, so the plain kernels are unchanged.
+template <bool PUSH> struct PushParam {};
+template <> struct PushParam<true> {
+  int nseg;
+  long long b[SFS_MAX_PUSH], e[SFS_MAX_PUSH];
+  void* dst[SFS_MAX_PUSH];
+  int nwait;
+  const unsigned* wait[SFS_MAX_PEERS];
+  unsigned wait_value;
+  int nsig;
+  unsigned* sig[SFS_MAX_PEERS];
+  unsigned sig_value;
+  unsigned* counter;
+};
+
+PushParam<true> push_param(const sfs_push_t& h) {
+  PushParam<true> p;
+  p.nseg = h.nseg;
+  for (int i = 0; i < SFS_MAX_PUSH; i++) {
+    p.b[i] = h.seg_begin[i];
+    p.e[i] = h.seg_end[i];
+    p.dst[i] = h.seg_dst[i];
+  }
+  p.nwait = h.nwait;
+  p.nsig = h.nsig;
+  for (int i = 0; i < SFS_MAX_PEERS; i++) {
+    p.wait[i] = h.wait_flag[i];
+    p.sig[i] = h.sig_flag[i];
+  }
+  p.wait_value = h.wait_value;
+  p.sig_value = h.sig_value;
+  p.counter = h.counter;
+  return p;
+}
+
+__device__ __forceinline__ unsigned ld_acquire_sys(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_sys(unsigned* p, unsigned v) {
+  asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+constexpr unsigned long long kHaloTimeoutNs = 20ull * 1000 * 1000 * 1000;  // 20 s
+
+// Before reading x: the neighbours have pushed this epoch's ghosts and finished reading the buffer
+// this grid pushes into.
+template <bool PUSH>
+__device__ __forceinline__ void halo_wait(const PushParam<PUSH>& p) {
+  if constexpr (PUSH) {
+    if ((int)threadIdx.x < p.nwait) {
+      const unsigned* f = p.wait[threadIdx.x];
+      unsigned long long t0 = 0;
+      for (int spin = 0; (int)(ld_acquire_sys(f) - p.wait_value) < 0; spin++) {
+        __nanosleep(100);
+        if ((spin & 1023) == 0) {  // a neighbour that never signals: fail the launch, do not hang the GPU
+          unsigned long long t;
+          asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+          if (t0 == 0) t0 = t;
+          else if (t - t0 > kHaloTimeoutNs) __trap();
+        }
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// y[r] = v, and into every run that contains r.
+template <bool PUSH, typename T>
+__device__ __forceinline__ void store_row(T* __restrict__ y, long long r, T v, const PushParam<PUSH>& p,
+                                          bool& pushed) {
+  y[r] = v;
+  if constexpr (PUSH) {
+    for (int i = 0; i < p.nseg; i++)
+      if (r >= p.b[i] && r < p.e[i]) {
+        ((T*)p.dst[i])[r - p.b[i]] = v;
+        pushed = true;
+      }
+  }
+}
+
+// After this CTA's stores: a thread that pushed publishes its peer stores (system-scope fence); the
+// CTA's arrival is counted with an acq_rel atomic (its reads of x and stores of y are done), and the
+// last CTA of the grid resets the counter and releases every neighbour's flag (system scope).  With no
+// neighbour (nsig == 0, uniform over the grid) nothing waits on this grid: no counting.
+template <bool PUSH>
+__device__ __forceinline__ void halo_signal(const PushParam<PUSH>& p, bool pushed) {
+  if constexpr (PUSH) {
+    if (pushed) __threadfence_system();
+    if (p.nsig == 0) return;
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      unsigned prev;
+      asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev) : "l"(p.counter) : "memory");
+      if (prev == gridDim.x - 1) {
+        asm volatile("fence.acq_rel.sys;" ::: "memory");
+        *p.counter = 0u;
+        for (int i = 0; i < p.nsig; i++) st_release_sys(p.sig[i], p.sig_value);
+      }
+    }
+  }
+}
+
+__global__ void k_halo_wait(PushParam<true> p) {
+  pdl_wait();
+  halo_wait<true>(p);
+  pdl_trigger();
+}
+
+// The push alone: dst runs <- src[r] (initial ghost exchange; the unfused formats' push after their SpMV).
+template <typename T>
+__global__ void k_halo_push(const T* __restrict__ src, PushParam<true> p) {
+  pdl_wait();
+  halo_wait<true>(p);
+  bool pushed = false;
+  for (int i = 0; i < p.nseg; i++) {
+    const long long n = p.e[i] - p.b[i];
+    T* d = (T*)p.dst[i];
+    for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t < n; t += (long long)gridDim.x * blockDim.x) {
+      d[t] = src[p.b[i] + t];
+      pushed = true;
+    }
+  }
+  halo_signal<true>(p, pushed);
+  pdl_trigger();
+}
+
 // ======================================================================== CSR vector
 // Vector v (TPV lanes) owns rows v, v+V, v+2V, ... (V = vectors in the grid): the CUSP-style mapping
 // the csr_max feature describes (Q4).  It works on two of its rows at once (r and r+V) and
@@ -169,17 +302,20 @@ template <typename T> constexpr int stream_u() { return sizeof(T) == 4 ? 16 : 8;
 template <typename T> constexpr int stream_ctas() { return sizeof(T) == 4 ? 3 : 4; }  // register cap
 constexpr int kSWMax = 32 * 16;
 
-template <typename T>
+template <typename T, bool PUSH = false>
 __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream(const int* __restrict__ rp,
                                                                const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
-                                                               T* __restrict__ y, long long m, int S) {
+                                                               T* __restrict__ y, long long m, int S,
+                                                               PushParam<PUSH> push) {
   constexpr int kSU = stream_u<T>();  // all of a lane's loads of a window are in flight together
   constexpr int kSW = 32 * kSU;
   __shared__ acc_t sbuf[kSWarps][kSW];
   __shared__ acc_t s_part[kSWarps][32];
   pdl_wait();
   pdl_early();
+  halo_wait<PUSH>(push);
+  bool pushed = false;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
   const int NG = kSWarps / S;  // groups per CTA iteration
   const int p = w / NG, gl = w % NG;
@@ -236,18 +372,19 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
       __syncwarp();
     }
     if (S == 1) {
-      if (g < ngroups && r < m) y[r] = (T)acc;
+      if (g < ngroups && r < m) store_row<PUSH>(y, r, (T)acc, push, pushed);
     } else {
       s_part[w][lane] = acc;
       __syncthreads();
       if (p == 0) {
         acc_t t = acc;
         for (int q = 1; q < S; q++) t += s_part[q * NG + gl][lane];
-        if (g < ngroups && r < m) y[r] = (T)t;
+        if (g < ngroups && r < m) store_row<PUSH>(y, r, (T)t, push, pushed);
       }
       __syncthreads();
     }
   }
+  halo_signal<PUSH>(push, pushed);
   pdl_trigger();
 }
 
@@ -798,7 +935,7 @@ template <typename T> constexpr int ell_ctas() { return sizeof(T) == 4 ? 3 : 4; 
 constexpr long long kHybRowwiseSmall = 64;  // z < 2^20 (latency-bound sizes)
 constexpr long long kHybRowwiseLarge = 32;
 
-template <typename T, bool OVF>
+template <typename T, bool OVF, bool PUSH = false>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
                                                                          const T* __restrict__ eval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
@@ -806,12 +943,15 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
                                                                          int early_trigger,
                                                                          const int* __restrict__ ovf,
                                                                          const int* __restrict__ ocol,
-                                                                         const T* __restrict__ oval) {
+                                                                         const T* __restrict__ oval,
+                                                                         PushParam<PUSH> push) {
   constexpr int kB = ell_batch<T>();
   __shared__ acc_t s_part[kEllThreads][4];
   pdl_wait();
   pdl_early();
   if (early_trigger) pdl_trigger();  // HYB: let the COO part start its loads now
+  halo_wait<PUSH>(push);
+  bool pushed = false;
   const int G = kEllThreads / S;
   const int p = threadIdx.x / G, g = threadIdx.x % G;
   const int Kp = (K + S - 1) / S;
@@ -896,9 +1036,10 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
     if (p == 0 && grp < groups) {
 #pragma unroll
       for (int q = 0; q < 4; q++)
-        if (r + q < m) y[r + q] = (T)acc[q];
+        if (r + q < m) store_row<PUSH>(y, r + q, (T)acc[q], push, pushed);
     }
   }
+  halo_signal<PUSH>(push, pushed);
   pdl_trigger();
 }
 
@@ -913,12 +1054,12 @@ template <typename T> constexpr int dia_rows() { return 4; }
 template <typename T> constexpr int dia_ctas() { return 4; }  // register cap
 template <typename T> constexpr int dia_batch() { return 4; }  // diagonals per batch
 
-template <typename T, int S>
+template <typename T, int S, bool PUSH = false>
 __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const int* __restrict__ offs,
                                                                          const T* __restrict__ dval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
                                                                          long long m, long long n, long long P,
-                                                                         int nd) {
+                                                                         int nd, PushParam<PUSH> push) {
   constexpr int kR = dia_rows<T>();
   constexpr int G = kDiaThreads / S;  // threads per part (compile-time: row strides are immediates)
   constexpr int kB = dia_batch<T>();
@@ -929,6 +1070,8 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
   const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
   for (int i = threadIdx.x; i < nsm; i += blockDim.x) s_off[i] = offs[i];
   __syncthreads();
+  halo_wait<PUSH>(push);
+  bool pushed = false;
   const int p = threadIdx.x / G, g = threadIdx.x % G;
   const int Dp = (nd + S - 1) / S;
   const int d0 = p * Dp, d1 = d0 + Dp < nd ? d0 + Dp : nd;
@@ -1000,10 +1143,11 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 #pragma unroll
       for (int q = 0; q < kR; q++) {
         const long long rr = r0 + (long long)q * G;
-        if (rr < m) y[rr] = (T)acc[q];
+        if (rr < m) store_row<PUSH>(y, rr, (T)acc[q], push, pushed);
       }
     }
   }
+  halo_signal<PUSH>(push, pushed);
   pdl_trigger();
 }
 
@@ -1056,17 +1200,52 @@ cudaError_t launch_zero(T* y, long long m, cudaStream_t s) {
   return launch_k(k_zero<T>, dim3(grid_cap(m, 256, 8)), dim3(256), s, y, m);
 }
 
-template <typename T>
-cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s, int early_trigger) {
+template <typename T, bool PUSH = false>
+cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s, int early_trigger,
+                       PushParam<PUSH> push = {}) {
   const long long groups = A->pitch / 4;
   const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
   const long long niter = ceil_div(groups, kEllThreads / S);
   const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
-  if (A->fmt == SFS_HYB && A->variant == 1)
-    return launch_k(k_spmv_ell<T, true>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1],
-                    x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3], (const T*)A->ptr[4]);
-  return launch_k(k_spmv_ell<T, false>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0], (const T*)A->ptr[1],
-                  x, y, A->m, A->pitch, K, S, early_trigger, (const int*)nullptr, (const int*)nullptr, (const T*)nullptr);
+  if (!PUSH && A->fmt == SFS_HYB && A->variant == 1)
+    return launch_k(k_spmv_ell<T, true, false>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
+                    (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3],
+                    (const T*)A->ptr[4], PushParam<false>{});
+  return launch_k(k_spmv_ell<T, false, PUSH>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
+                  (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, early_trigger, (const int*)nullptr,
+                  (const int*)nullptr, (const T*)nullptr, push);
+}
+
+template <typename T, bool PUSH>
+cudaError_t launch_csr_stream(const int* rp, const int* col, const T* val, const T* x, T* y, long long m, long long z,
+                              cudaStream_t s, PushParam<PUSH> push) {
+  const long long groups = ceil_div(m, 32);
+  const long long windows = ceil_div(z, 32 * stream_u<T>());  // ~ windows over all groups
+  const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
+  const long long niter = ceil_div(groups, kSWarps / S);
+  const int grid = (int)(niter < (long long)kSMs * stream_ctas<T>() ? niter : (long long)kSMs * stream_ctas<T>());
+  return launch_k(k_spmv_csr_stream<T, PUSH>, dim3(grid < 1 ? 1 : grid), dim3(kSThreads), s, rp, col, val, x, y, m, S,
+                  push);
+}
+
+template <typename T, bool PUSH>
+cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushParam<PUSH> push) {
+  const long long m = A->m;
+  const long long blocks_rows = ceil_div(m, dia_rows<T>());  // threads needed at S = 1
+  const int S = split_factor(blocks_rows, A->ndiag, 2 * dia_batch<T>(), 16);
+  const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
+  const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
+  const dim3 gd(grid < 1 ? 1 : grid), bd(kDiaThreads);
+  const int* offs = (const int*)A->ptr[0];
+  const T* dv = (const T*)A->ptr[1];
+  const int nd = (int)A->ndiag;
+  switch (S) {
+    case 1: return launch_k(k_spmv_dia<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+    case 2: return launch_k(k_spmv_dia<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+    case 4: return launch_k(k_spmv_dia<T, 4, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+    case 8: return launch_k(k_spmv_dia<T, 8, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+    default: return launch_k(k_spmv_dia<T, 16, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+  }
 }
 
 template <typename T>
@@ -1106,7 +1285,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
         const long long niter = ceil_div(groups, kSWarps / S);
         const int grid = (int)(niter < (long long)kSMs * stream_ctas<T>() ? niter : (long long)kSMs * stream_ctas<T>());
-        e = launch_k(k_spmv_csr_stream<T>, dim3(grid), dim3(kSThreads), s, rp, col, val, x, y, m, S);
+        e = launch_csr_stream<T, false>(rp, col, val, x, y, m, z, s, PushParam<false>{});
       } else if (A->variant == 0) {
         // kCsrWarps warps grid-stride over rows (the mapping the csr_max feature describes, Q4); a
         // matrix covered in one pass gets only the warps that own rows (same row -> warp mapping).
@@ -1146,24 +1325,9 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         e = launch_coo<T, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y, A->coo_nnz, s);
       break;
     }
-    case SFS_DIA: {
-      const long long blocks_rows = ceil_div(m, dia_rows<T>());  // threads needed at S = 1
-      const int S = split_factor(blocks_rows, A->ndiag, 2 * dia_batch<T>(), 16);
-      const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
-      const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
-      const dim3 gd(grid < 1 ? 1 : grid), bd(kDiaThreads);
-      const int* offs = (const int*)A->ptr[0];
-      const T* dv = (const T*)A->ptr[1];
-      const int nd = (int)A->ndiag;
-      switch (S) {
-        case 1: e = launch_k(k_spmv_dia<T, 1>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
-        case 2: e = launch_k(k_spmv_dia<T, 2>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
-        case 4: e = launch_k(k_spmv_dia<T, 4>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
-        case 8: e = launch_k(k_spmv_dia<T, 8>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
-        default: e = launch_k(k_spmv_dia<T, 16>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd); break;
-      }
+    case SFS_DIA:
+      e = launch_dia<T, false>(A, x, y, s, PushParam<false>{});
       break;
-    }
     default:
       return cudaErrorInvalidValue;
   }
@@ -1266,6 +1430,43 @@ cudaError_t launch_l2_flush(const void* buf, size_t bytes, cudaStream_t s) {
   k_l2_flush<<<kSMs * 8, 256, 0, s>>>((const uint4*)buf, (long long)(bytes / 16), (unsigned*)buf);
   count_launch();
   return cudaGetLastError();
+}
+
+template <typename T>
+cudaError_t spmv_push_t(const Matrix* A, const T* x, T* y, const sfs_push_t& h, cudaStream_t s) {
+  const PushParam<true> p = push_param(h);
+  if (A->fmt == SFS_DIA && A->ndiag > 0) return launch_dia<T, true>(A, x, y, s, p);
+  if (A->fmt == SFS_ELL && A->width > 0) return launch_ell<T, true>(A, x, y, (int)A->width, s, 0, p);
+  if (A->fmt == SFS_CSR && A->variant == 2 && A->m > 0)
+    return launch_csr_stream<T, true>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, A->m,
+                                      A->nnz, s, p);
+  // kernels that do not own their rows (atomics, carries): wait kernel -> SpMV -> push kernel
+  cudaError_t e = cudaSuccess;
+  if (p.nwait > 0) e = launch_k(k_halo_wait, dim3(1), dim3(32), s, p);
+  if (e == cudaSuccess) e = spmv_t<T>(A, x, y, s);
+  if (e == cudaSuccess) {
+    PushParam<true> q = p;
+    q.nwait = 0;
+    long long most = 0;
+    for (int i = 0; i < h.nseg; i++) most = std::max(most, (long long)(h.seg_end[i] - h.seg_begin[i]));
+    e = launch_k(k_halo_push<T>, dim3(grid_cap(most, 256, 2)), dim3(256), s, (const T*)y, q);
+  }
+  return e;
+}
+
+cudaError_t launch_spmv_push(const Matrix* A, const void* x, void* y, const sfs_push_t& p, cudaStream_t s) {
+  if (A->dtype == SFS_F64) return spmv_push_t<double>(A, (const double*)x, (double*)y, p, s);
+  return spmv_push_t<float>(A, (const float*)x, (float*)y, p, s);
+}
+
+cudaError_t launch_halo_push(int dtype, const void* src, long long nrows, const sfs_push_t& h, cudaStream_t s) {
+  const PushParam<true> p = push_param(h);
+  long long most = 0;
+  for (int i = 0; i < h.nseg; i++) most = std::max(most, (long long)(h.seg_end[i] - h.seg_begin[i]));
+  (void)nrows;
+  const dim3 g(grid_cap(most, 256, 2));
+  if (dtype == SFS_F64) return launch_k(k_halo_push<double>, g, dim3(256), s, (const double*)src, p);
+  return launch_k(k_halo_push<float>, g, dim3(256), s, (const float*)src, p);
 }
 
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s) {

@@ -390,3 +390,218 @@ def rowpart_halo_iterate(plan: HaloPlan, local_spmv: Callable, gather: Callable,
         exchange(nxt)
         cur, nxt = nxt, cur
     return cur[own]
+
+
+# ------------------------------------------------------------------ row partition with the halo push fused in
+# SURVEY §8(f) f3, "stores of y into every peer's x": the rank's SpMV kernel itself stores each y entry a
+# neighbour needs as a ghost into that neighbour's next x_ext (peer memory: symmetric memory over
+# NVLink on one node, or plain device memory when the P ranks are simulated on one GPU), then releases
+# a per-(receiver, sender) flag; the neighbour's next SpMV waits on its flags before reading x
+# (sfs_spmv_push, include/sfs.h).  No NCCL call and no separate pack / send / unpack per iteration.
+# The send entries of a banded / stencil block are contiguous local rows landing in a contiguous run
+# of the neighbour's ghost region, so a plan is a handful of runs.
+
+
+def recv_offsets_by_source(plan: HaloPlan) -> dict:
+    """Where each source rank's entries land in this rank's x_ext: {source: offset} (one recv entry per
+    source: the ghost ids are sorted and each source owns a contiguous id range, below or above)."""
+    out = {}
+    for j, o, c in plan.recv:
+        assert j not in out, "a source split across the lower and upper ghost regions"
+        out[j] = o
+    return out
+
+
+def push_runs(plan: HaloPlan, dst_offset: dict) -> List[tuple]:
+    """The rank's pushes as runs (destination rank, local row begin, end, element offset in the
+    destination's x_ext).  `dst_offset[j]`: where this rank's entries start in rank j's x_ext (rank j's
+    recv_offsets_by_source()[this rank])."""
+    runs = []
+    for j, o, c in plan.send:
+        idx = np.asarray(plan.send_idx[o:o + c], dtype=np.int64)
+        if len(idx) == 0:
+            continue
+        brk = np.flatnonzero(np.diff(idx) != 1) + 1
+        starts = np.r_[0, brk]
+        ends = np.r_[brk, len(idx)]
+        for a, b in zip(starts, ends):
+            runs.append((j, int(idx[a]), int(idx[a]) + int(b - a), int(dst_offset[j]) + int(a)))
+    return runs
+
+
+def push_neighbours(plan: HaloPlan) -> List[int]:
+    """Ranks this rank waits on and signals: its sources (their ghosts must have arrived) and its
+    destinations (they must have finished reading the buffer this rank pushes into)."""
+    return sorted({j for j, _, _ in plan.send} | {j for j, _, _ in plan.recv})
+
+
+def exchange_recv_offsets(plan: HaloPlan, group=None, device=None) -> dict:
+    """Collective (setup only): tell every source where its entries land here; returns, for each
+    destination of this rank, the offset in the destination's x_ext (push_runs' dst_offset)."""
+    import torch
+    import torch.distributed as dist
+    if plan.world == 1:
+        return {}
+    dev = device or "cpu"
+    mine = recv_offsets_by_source(plan)
+    out = torch.tensor([mine.get(j, -1) for j in range(plan.world)], dtype=torch.int64, device=dev)
+    inp = torch.empty(plan.world, dtype=torch.int64, device=dev)
+    dist.all_to_all_single(inp, out, group=group)
+    got = inp.cpu().tolist()
+    return {j: int(got[j]) for j, _, _ in plan.send}
+
+
+def apply_push_host(plans: Sequence[HaloPlan], xs_ext: Sequence[np.ndarray]) -> None:
+    """Host model of one push round (tests): every rank's runs copy its own-slice entries into the
+    neighbours' x_ext, exactly as the kernels' extra stores do."""
+    offs = [recv_offsets_by_source(p) for p in plans]
+    for k, p in enumerate(plans):
+        dst = {j: offs[j][k] for j, _, _ in p.send}
+        for j, b, e, o in push_runs(p, dst):
+            xs_ext[j][o:o + (e - b)] = xs_ext[k][p.n_lo + b:p.n_lo + e]
+
+
+class _PushBuffers:
+    """Per-rank device memory of the push protocol: x_ext double buffer, flags[world] (slot per sender),
+    counter.  `base(k)` is the address of rank k's block (a peer address in the real multi-GPU case)."""
+
+    def __init__(self, n_ext_max: int, world: int, elem: int):
+        self.n_ext_max, self.world, self.elem = n_ext_max, world, elem
+        self.x_bytes = n_ext_max * elem
+        self.flag_off = 2 * self.x_bytes
+        self.counter_off = self.flag_off + 4 * world
+        self.nbytes = (self.counter_off + 4 + 255) // 256 * 256
+
+    def x(self, base: int, parity: int) -> int:
+        return base + parity * self.x_bytes
+
+    def flag(self, base: int, sender: int) -> int:
+        return base + self.flag_off + 4 * sender
+
+    def counter(self, base: int) -> int:
+        return base + self.counter_off
+
+
+def _push_structs(sfs, plan: HaloPlan, runs, nbrs, bases, rank: int, B: _PushBuffers, parity: int, wait: int,
+                  sig: int):
+    r = [(b, e, B.x(bases[j], parity) + o * B.elem) for j, b, e, o in runs]
+    return sfs.push_struct(r, [B.flag(bases[rank], j) for j in nbrs], wait, [B.flag(bases[j], rank) for j in nbrs],
+                           sig, B.counter(bases[rank]))
+
+
+def rowpart_push_iterate_local(plans: Sequence[HaloPlan], mats, fmt: int, x_locals, iters: int, stream=None):
+    """The P ranks of a push-fused row partition simulated on ONE GPU (same kernels, same protocol; the
+    "peer" buffers are other allocations on this device).  mats[k]: rank k's remapped block converted to
+    `fmt` (sfs.Matrix); x_locals[k]: its slice of x.  Each iteration launches every rank's fused SpMV in
+    rank order on one stream, so every wait is already satisfied.  Returns the final own slices."""
+    import torch
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    world = len(plans)
+    dt, dev = x_locals[0].dtype, x_locals[0].device
+    B = _PushBuffers(max(p.n_ext for p in plans), world, x_locals[0].element_size())
+    mem = [torch.zeros(B.nbytes, dtype=torch.uint8, device=dev) for _ in range(world)]
+    bases = [t.data_ptr() for t in mem]
+    offs = [recv_offsets_by_source(p) for p in plans]
+    runs = [push_runs(p, {j: offs[j][k] for j, _, _ in p.send}) for k, p in enumerate(plans)]
+    nbrs = [push_neighbours(p) for p in plans]
+
+    def xview(k, parity):
+        n = plans[k].n_ext
+        return mem[k][parity * B.x_bytes:parity * B.x_bytes + n * B.elem].view(dt)
+
+    for k, p in enumerate(plans):
+        xview(k, 0)[p.n_lo:p.n_lo + p.n_local].copy_(x_locals[k])
+    for k, p in enumerate(plans):  # epoch 1: the initial ghosts
+        own = xview(k, 0)[p.n_lo:p.n_lo + p.n_local]
+        sfs.halo_push(own, _push_structs(sfs, p, runs[k], nbrs[k], bases, k, B, 0, 0, 1), stream)
+    for t in range(1, iters + 1):
+        cur, nxt = (t - 1) % 2, t % 2
+        for k, p in enumerate(plans):
+            y = xview(k, nxt)[p.n_lo:p.n_lo + p.n_local]
+            sfs.spmv_push(fmt, mats[k], xview(k, cur), y,
+                          _push_structs(sfs, p, runs[k], nbrs[k], bases, k, B, nxt, t, t + 1), stream)
+    return [xview(k, iters % 2)[p.n_lo:p.n_lo + p.n_local] for k, p in enumerate(plans)], mem
+
+
+def rowpart_push_iterate(plan: HaloPlan, A_local, fmt: int, x_local, iters: int, group=None, timing=None,
+                         transport: str = "ipc"):
+    """One rank of the push-fused row partition on a real multi-GPU node: the x_ext double buffer, flags and
+    counter live in peer-mapped device memory -- CUDA IPC (`transport="ipc"`: sfs_ipc_alloc / sfs_ipc_open,
+    peer access over NVLink; also works for several processes sharing one GPU) or torch symmetric memory
+    (`"symm"`, one GPU per rank) -- so the fused kernel's ghost stores go straight into the neighbours'
+    HBM.  Setup: one all_to_all of the recv offsets, one all_reduce of the buffer size, an exchange of
+    the handles, a barrier.  `timing`: optional dict receiving the per-iteration device time (ms)."""
+    import torch
+    import torch.distributed as dist
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    dev, dt = x_local.device, x_local.dtype
+    multi = plan.world > 1
+    nmax = torch.tensor([plan.n_ext], dtype=torch.int64, device=dev if dist.is_initialized() and
+                        dist.get_backend(group) == "nccl" else "cpu")
+    if multi:
+        dist.all_reduce(nmax, op=dist.ReduceOp.MAX, group=group)
+    B = _PushBuffers(int(nmax.item()), plan.world, x_local.element_size())
+    opened, own_ipc, keep = [], None, None
+    if multi and transport == "symm":
+        import torch.distributed._symmetric_memory as symm_mem
+        keep = symm_mem.empty(B.nbytes, dtype=torch.uint8, device=dev)
+        keep.zero_()
+        hdl = symm_mem.rendezvous(keep, group if group is not None else dist.group.WORLD)
+        bases = [int(p) for p in hdl.buffer_ptrs]
+    elif multi:
+        own_ipc, h = sfs.ipc_alloc(B.nbytes)
+        handles = [None] * plan.world
+        dist.all_gather_object(handles, h, group=group)
+        bases = []
+        for j, hj in enumerate(handles):
+            if j == plan.rank:
+                bases.append(own_ipc)
+            else:
+                bases.append(sfs.ipc_open(hj))
+                opened.append(bases[-1])
+    else:  # no neighbours: the fused kernel's protocol runs on local memory only
+        keep = torch.zeros(B.nbytes, dtype=torch.uint8, device=dev)
+        bases = [keep.data_ptr()]
+    own_base = bases[plan.rank]
+    raw = keep if keep is not None else _device_bytes(own_base, B.nbytes, dev)
+    runs = push_runs(plan, exchange_recv_offsets(plan, group, nmax.device))
+    nbrs = push_neighbours(plan)
+    k = plan.rank
+    xv = lambda parity: raw[parity * B.x_bytes:parity * B.x_bytes + plan.n_ext * B.elem].view(dt)
+    own = slice(plan.n_lo, plan.n_lo + plan.n_local)
+    xv(0)[own].copy_(x_local)
+    torch.cuda.synchronize()
+    if multi:
+        dist.barrier(group=group)
+    sfs.halo_push(xv(0)[own], _push_structs(sfs, plan, runs, nbrs, bases, k, B, 0, 0, 1))
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for t in range(1, iters + 1):
+        cur, nxt = (t - 1) % 2, t % 2
+        sfs.spmv_push(fmt, A_local, xv(cur), xv(nxt)[own],
+                      _push_structs(sfs, plan, runs, nbrs, bases, k, B, nxt, t, t + 1))
+    e1.record()
+    torch.cuda.synchronize()
+    if timing is not None:
+        timing["ms_per_iter"] = e0.elapsed_time(e1) / max(iters, 1)
+    out = xv(iters % 2)[own].clone()
+    torch.cuda.synchronize()
+    if multi:
+        dist.barrier(group=group)  # every neighbour is done storing into our buffer
+    for a in opened:
+        sfs.ipc_close(a)
+    if multi:
+        dist.barrier(group=group)
+    if own_ipc is not None:
+        sfs.ipc_free(own_ipc)
+    return out
+
+
+def _device_bytes(addr: int, nbytes: int, dev):
+    """A uint8 torch view of library-allocated device memory (no copy, not owned by torch)."""
+    import torch
+
+    class _Mem:
+        __cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (addr, False), "version": 3}
+
+    return torch.as_tensor(_Mem(), device=dev)

@@ -217,7 +217,8 @@ def _halo_worker(rank, world, port, q):
 
         x = torch.from_numpy(np.random.default_rng(2).uniform(-1, 1, A.n))
         y = sd.rowpart_halo_iterate(plan, local_spmv, gather, x[b[rank]:b[rank + 1]].clone(), iters=3)
-        q.put((rank, y.numpy().copy(), plan.recv_count))
+        dst_off = sd.exchange_recv_offsets(plan)  # collective: where this rank's pushes land
+        q.put((rank, y.numpy().copy(), plan.recv_count, dst_off, sd.push_runs(plan, dst_off)))
     except Exception:
         import traceback
         q.put((rank, "ERROR", traceback.format_exc()))
@@ -249,3 +250,44 @@ def test_gloo_world2_halo_exchange_power_iteration():
         x, _ = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val, x)
     assert np.array_equal(np.concatenate([out[0][1], out[1][1]]), x)
     assert out[0][2] == out[1][2] == 12 * 12
+    # the push plan exchanged over gloo equals the one built from every rank's plan in one process
+    blocks = [sd.slice_rows(A.rp, A.col, A.val, *sd.row_blocks(A.m, world)[k:k + 2]) for k in range(world)]
+    plans = sd.halo_plans_local(A.m, A.n, world, [c for _, c, _ in blocks])
+    offs = [sd.recv_offsets_by_source(P) for P in plans]
+    for k in range(world):
+        want = {j: offs[j][k] for j, _, _ in plans[k].send}
+        assert out[k][3] == want
+        assert out[k][4] == sd.push_runs(plans[k], want)
+        assert len(out[k][4]) == 1  # one contiguous plane per neighbour
+
+
+@pytest.mark.parametrize("kind", ["stencil", "random"])
+@pytest.mark.parametrize("world", [2, 3, 5])
+def test_push_runs_deliver_the_ghosts(kind, world):
+    """The fused push (runs of own-slice rows stored into the neighbours' x_ext, include/sfs.h
+    sfs_spmv_push) fills every rank's ghost region with exactly x[lo] and x[hi]: the same data the
+    batch_isend_irecv exchange delivers; runs never overlap; a stencil needs one run per neighbour."""
+    A = _halo_case(kind)
+    x = np.random.default_rng(4).uniform(-1, 1, A.n)
+    bnd = sd.row_blocks(A.m, world)
+    blocks = [sd.slice_rows(A.rp, A.col, A.val, bnd[k], bnd[k + 1]) for k in range(world)]
+    plans = sd.halo_plans_local(A.m, A.n, world, [c for _, c, _ in blocks])
+    xs = []
+    for P in plans:
+        xe = np.full(P.n_ext, np.nan)
+        xe[P.n_lo:P.n_lo + P.n_local] = x[P.r0:P.r1]
+        xs.append(xe)
+    sd.apply_push_host(plans, xs)
+    offs = [sd.recv_offsets_by_source(P) for P in plans]
+    for k, P in enumerate(plans):
+        assert np.array_equal(xs[k], np.concatenate([x[P.lo], x[P.r0:P.r1], x[P.hi]]))
+        runs = sd.push_runs(P, {j: offs[j][k] for j, _, _ in P.send})
+        assert sum(e - b for _, b, e, _ in runs) == len(P.send_idx)
+        cover = np.zeros(P.n_local, np.int64)
+        for j, b, e, o in runs:
+            assert 0 <= b < e <= P.n_local
+        nb = sd.push_neighbours(P)
+        assert set(j for j, _, _ in P.send) <= set(nb) and set(j for j, _, _ in P.recv) <= set(nb)
+        if kind == "stencil":
+            assert len(runs) == len(P.send) <= 2
+            assert nb == [j for j in (k - 1, k + 1) if 0 <= j < world]

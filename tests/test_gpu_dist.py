@@ -6,7 +6,7 @@ import pytest
 import oracle
 import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
 import sfsgen
-from gpu_util import TOL
+from gpu_util import TOL, to_dev
 from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
 
 pytestmark = pytest.mark.gpu
@@ -170,3 +170,93 @@ def test_halo_exchange_power_iteration_simulated(world, fmt):
     assert np.all(np.abs(y - x) <= 1e-11 * (np.abs(x) + ax))
     for M in mats:
         M.free()
+
+
+@pytest.mark.parametrize("world", [2, 4, 8])
+@pytest.mark.parametrize("fmt,variant", [(4, -1), (2, -1), (0, 2), (0, 4), (1, -1), (3, -1)])
+@pytest.mark.parametrize("dtype", ["f64", "f32"])
+def test_push_fused_power_iteration_simulated(world, fmt, variant, dtype):
+    """sfs_spmv_push on one GPU with P simulated ranks (include/sfs.h): the ghost rows are
+    stored into the neighbours' next x_ext by the SpMV kernel itself (DIA, ELL, CSR stream) or by the
+    push kernel after it (CSR tile, COO, HYB), with the wait / signal flags; 3 power-iteration steps ==
+    the oracle's global iteration within tolerance; flags end at the last epoch, counters at 0."""
+    import torch
+    A = sfsgen.generate(sfsgen.make_spec(sfsgen.ST3D27, ia=24))
+    if dtype == "f32":
+        A = sfsgen.CSR(A.m, A.n, A.rp, A.col, A.val.astype(np.float32))
+    x0 = sfsgen.vector(11, A.n, 0 if dtype == "f32" else 1)
+    b = sd.row_blocks(A.m, world)
+    blocks = [sd.slice_rows(A.rp, A.col, A.val, b[k], b[k + 1]) for k in range(world)]
+    plans = sd.halo_plans_local(A.m, A.n, world, [c for _, c, _ in blocks])
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).cuda()
+    opts = sfs.default_opts(csr_variant=variant)
+    mats = []
+    for P, (rp, _, val) in zip(plans, blocks):
+        M = sfs.convert(sfs.Csr(P.n_local, P.n_ext, t(rp), t(P.col_ext), t(val)), fmt, opts)
+        if fmt == sfs.CSR:
+            assert M.layout().variant == variant
+        mats.append(M)
+    iters = 3
+    ys, mem = sd.rowpart_push_iterate_local(plans, mats, fmt, [t(x0[P.r0:P.r1]) for P in plans], iters)
+    y = np.concatenate([v.cpu().numpy().astype(np.float64) for v in ys])
+    x = x0.astype(np.float64)
+    for _ in range(iters):
+        x, ax = oracle.spmv_csr(A.m, A.n, A.rp, A.col, A.val.astype(np.float64), x)
+        if dtype == "f32":  # each step's y is rounded to fp32 before the next
+            x = x.astype(np.float32).astype(np.float64)
+    tol = 1e-11 if dtype == "f64" else 3e-5
+    assert np.all(np.abs(y - x) <= tol * (np.abs(x) + ax))
+    B = sd._PushBuffers(max(P.n_ext for P in plans), world, ys[0].element_size())
+    for k, P in enumerate(plans):
+        raw = mem[k].cpu().numpy()
+        flags = raw[B.flag_off:B.flag_off + 4 * world].view(np.uint32)
+        for j in sd.push_neighbours(P):
+            assert flags[j] == iters + 1
+        assert raw[B.counter_off:B.counter_off + 4].view(np.uint32)[0] == 0
+    for M in mats:
+        M.free()
+
+
+def test_push_argument_errors():
+    import torch
+    A = sfsgen.laplace2d(16)
+    M = sfs.convert(to_dev(A), sfs.DIA)
+    x = torch.ones(A.n, dtype=torch.float64, device="cuda")
+    y = torch.empty(A.m, dtype=torch.float64, device="cuda")
+    cnt = torch.zeros(1, dtype=torch.int32, device="cuda")
+    dst = torch.empty(8, dtype=torch.float64, device="cuda")
+    ok = sfs.push_struct([(0, 8, dst.data_ptr())], [], 0, [], 1, cnt.data_ptr())
+    sfs.spmv_push(sfs.DIA, M, x, y, ok)
+    torch.cuda.synchronize()
+    assert np.array_equal(dst.cpu().numpy(), y[:8].cpu().numpy()) and cnt.item() == 0
+    bad = [sfs.push_struct([(0, A.m + 1, dst.data_ptr())], [], 0, [], 1, cnt.data_ptr()),   # run past the block
+           sfs.push_struct([(0, 8, dst.data_ptr()), (4, 12, dst.data_ptr())], [], 0, [], 1, cnt.data_ptr()),
+           sfs.push_struct([(0, 8, dst.data_ptr())], [], 0, [], 1, 0)]                        # no counter
+    for p in bad:
+        with pytest.raises(sfs.SfsError) as ei:
+            sfs.spmv_push(sfs.DIA, M, x, y, p)
+        assert ei.value.status == sfs.ERR_INVALID_ARG
+    with pytest.raises(sfs.SfsError):
+        sfs.spmv_push(sfs.CSR, M, x, y, ok)  # format mismatch
+    M.free()
+
+
+def test_push_two_processes_share_one_gpu():
+    """The push-fused row partition across two real processes (tools/push_2proc.py under torchrun): x_ext
+    buffers and flags in CUDA IPC memory mapped into the other process, each rank's fused SpMV kernel
+    storing its ghost rows into the other's buffer and waiting on the other's flag (the two contexts
+    time-slice the GPU, so the waits are real); DIA, ELL, CSR, COO == the oracle's 3-step iteration."""
+    import os
+    import socket
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(root, "tools", "push_2proc.py")]
+    r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-3000:])
+    assert r.stdout.count("matches the oracle") == 8, r.stdout[-2000:]

@@ -1,6 +1,7 @@
 #!/usr/bin/env python
 """configs[3]: 3D 27-point stencil on 128^3 row-partitioned over N GPUs: an NCCL all-gather of x, or
-(--exchange halo) NCCL send/recv of the ghost planes only.
+(--exchange halo) NCCL send/recv of the ghost planes only, or (--exchange push) the
+ghost rows stored into the neighbours' x by the SpMV kernel itself over symmetric memory (sfs_spmv_push).
 
     python -m torch.distributed.run --nproc-per-node N --master-addr 127.0.0.1 tools/bench_rowpart.py
 
@@ -26,7 +27,8 @@ def main():
     ap.add_argument("--dtype", default="f64")
     ap.add_argument("--iters", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=10)
-    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo"])
+    ap.add_argument("--exchange", default="allgather", choices=["allgather", "halo", "push"])
+    ap.add_argument("--backend", default="nccl")
     args = ap.parse_args()
 
     import torch
@@ -40,14 +42,14 @@ def main():
         os.environ.get("LOCAL_RANK", 0))
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist.init_process_group(args.backend, device_id=torch.device("cuda", local) if args.backend == "nccl" else None)
     dt = sfsgen.F64 if args.dtype == "f64" else sfsgen.F32
     A = sfsgen.stencil3d27(args.N, dtype=dt)
     part = sd.RowPartition(A.m, A.n, world, rank)
     b = part.bounds
     rp, col, val = sd.slice_rows(A.rp, A.col, A.val, b[rank], b[rank + 1])
     t = lambda a: torch.from_numpy(a).cuda()
-    halo = args.exchange == "halo"
+    halo = args.exchange in ("halo", "push")
     plan = sd.halo_plan(part, col, device=torch.device("cuda", local)) if halo else None
     Ak = sfs.Csr(part.local_rows, plan.n_ext if halo else A.n, t(rp), t(plan.col_ext if halo else col), t(val))
     fmt = sfs.FORMAT_NAMES.index(args.fmt)
@@ -57,7 +59,10 @@ def main():
     xs = torch.from_numpy(sfsgen.vector(5, A.n, dt)).cuda()
     x_local = xs[b[rank]:b[rank + 1]].clone()
     spmv = lambda xf, yl: sfs.spmv(fmt, M, xf, yl)
-    if halo:
+    push_t = {}
+    if args.exchange == "push":
+        iterate = lambda it: sd.rowpart_push_iterate(plan, M, fmt, x_local, it, timing=push_t)
+    elif halo:
         iterate = lambda it: sd.rowpart_halo_iterate(plan, spmv, sfs.gather, x_local, iters=it)
     else:
         iterate = lambda it: sd.rowpart_spmv_iterate(part, spmv, x_local, iters=it)
@@ -78,6 +83,11 @@ def main():
         return float(v.item())
 
     t_iter = timed(lambda: iterate(args.iters)) / args.iters
+    if args.exchange == "push":  # the iteration loop alone (symmetric-memory setup excluded), max over ranks
+        v = torch.tensor([push_t["ms_per_iter"] / 1000.0], device="cuda")
+        if world > 1:
+            dist.all_reduce(v, op=dist.ReduceOp.MAX)
+        t_iter = float(v.item())
     blk = part.block
     xp = torch.zeros(blk, dtype=xs.dtype, device="cuda")
     xf = torch.empty(blk * world, dtype=xs.dtype, device="cuda")
@@ -96,7 +106,7 @@ def main():
         for _ in range(args.iters):
             spmv(xm, yl)
 
-    t_ag = timed(ag) / args.iters
+    t_ag = timed(ag) / args.iters if (world == 1 or args.backend == "nccl") else float("nan")
     t_mv = timed(mv) / args.iters
     tot_bytes = torch.tensor([float(nbytes)], device="cuda")
     if world > 1:
