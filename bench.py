@@ -365,13 +365,29 @@ def run_ours(args):
                            f"part of each matrix from L2")
     except Exception:
         pass
+    l2 = None
+    try:  # the L2-sector view: gather-heavy SpMVs are bound by the SM <- L2 sector rate, not by HBM
+        with open(os.path.join(ROOT, "profiles", "r01", "ceilings.json")) as fh:
+            cj = json.load(fh)
+        with open(os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json")) as fh:
+            tj = json.load(fh).get(dom)
+        if tj and tj.get("l2_sectors_per_launch"):
+            rate = tj["l2_sectors_per_launch"] * launches_dom / per_fmt[dom]["spmv_time_s"] / 1e9
+            l2 = {"bound": "l2_sectors", "achieved": rate, "peak": cj["l2_random_sector_rate_gsps"],
+                  "unit": "G sectors/s", "frac": rate / cj["l2_random_sector_rate_gsps"],
+                  "sectors_per_launch": tj["l2_sectors_per_launch"],
+                  "source": "ncu lts__t_sectors_srcunit_tex.sum of the same kernels on this workload "
+                            "(profiles/r01/traffic_corpus200.json) over this run's event-timed race time; peak = "
+                            "measured random-sector rate of tools/gather.cu (profiles/r01/ceilings.txt)"}
+    except Exception:
+        pass
     step_time = t_dev / args.steps
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak if achieved else None, "traffic": traffic, "traffic_source": traffic_src,
                 "kernel": f"SpMV {dom}: {kernels[dom]}", "bytes_per_launch": bytes_per_launch,
                 "launches": launches_dom, "peak_source": peak_src,
                 "share_of_step": per_fmt[dom]["spmv_time_s"] / step_time,
-                "achieved_footprint_gt_2xL2": per_fmt[dom]["gbs_footprint_gt_2xL2"],
+                "achieved_footprint_gt_2xL2": per_fmt[dom]["gbs_footprint_gt_2xL2"], "l2": l2,
                 "note": "achieved = sum over the step's matrices of algorithmic bytes (SURVEY 8(a) a9-a13) x reps / "
                         "sum of their event-timed race time (CUDA events on the launching stream); reps run "
                         "back-to-back (P:L217), so the many corpus matrices that fit the 126 MB L2 are latency- "

@@ -1,6 +1,7 @@
 """Measured DRAM traffic per SpMV launch on the bench workload itself (corpus-200), per format.
 
-Input: an ncu CSV (--metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum
+Input: an ncu CSV (--metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum,
+lts__t_sectors_srcunit_tex.sum
 --cache-control none -k regex:"k_spmv|k_zero") of `bench.py --steps 1 --warmup 0 --reps R
 --race-warmup W --dump D`, and that dump.  The SpMV launches come in race order (matrix by matrix,
 formats CSR..DIA, W + R calls each); each call's kernels are predicted from the matrix's features
@@ -79,6 +80,7 @@ def main(csv_path, dump_path, calls, out=None):
                         a = acc[fmt]
                         a["dram"] += launches[pos].get("dram__bytes_read.sum", 0) + launches[pos].get("dram__bytes_write.sum", 0)
                         a["ns"] += launches[pos].get("gpu__time_duration.sum", 0)
+                        a["l2s"] += launches[pos].get("lts__t_sectors_srcunit_tex.sum", 0)
                     pos += 1
             acc[fmt]["alg"] += L["bytes"][fmt]
             acc[fmt]["n"] += 1
@@ -90,11 +92,13 @@ def main(csv_path, dump_path, calls, out=None):
         res[NAMES[fmt]] = {"launches": int(a["n"]), "dram_bytes_per_launch": a["dram"] / a["n"],
                            "algorithmic_bytes_per_launch": a["alg"] / a["n"], "ratio": a["dram"] / a["alg"],
                            "ncu_us_per_launch": a["ns"] / a["n"] / 1e3,
+                           "l2_sectors_per_launch": a["l2s"] / a["n"],
                            "kernel": "+".join(sorted({k for d in dump for k in kernels_of(fmt, d["features"], d["nnz"])}))}
     res["_source"] = {"csv": csv_path, "dump": dump_path, "calls_per_format": calls, "launches_parsed": pos,
                       "launches_in_csv": len(launches),
                       "note": "last of W+R back-to-back calls per (matrix, format), ncu --cache-control none: "
-                              "the hot-rep DRAM traffic of the race; per launch = averaged over the corpus"}
+                              "the hot-rep DRAM traffic of the race; per launch = averaged over the corpus; "
+                              "l2_sectors = lts__t_sectors_srcunit_tex.sum (32 B sectors the SMs requested from L2)"}
     s = json.dumps(res, indent=1)
     print(s)
     if out:
