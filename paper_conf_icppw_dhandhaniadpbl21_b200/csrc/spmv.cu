@@ -1005,8 +1005,15 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
 #pragma unroll
           for (int u = 0; u < 4; u++) {
             const int kk = k + u < ob[4] ? k + u : ob[4] - 1;
+#ifdef SFS_OVF_STREAM
             c[u] = ld_stream(ocol + kk);
             v[u] = ld_stream(oval + kk);
+#else
+            // L1-allocating: a thread's 4 consecutive entries share a sector, so the 2nd-4th loads hit
+            // L1 instead of each requesting the sector from L2 again (L2 sectors bound these SpMVs)
+            c[u] = __ldg(ocol + kk);
+            v[u] = __ldg(oval + kk);
+#endif
           }
 #pragma unroll
           for (int u = 0; u < 4; u++) {
