@@ -433,6 +433,11 @@ def run_ours(args):
 
 def main():
     args = parse()
+    # torchrun pins OMP_NUM_THREADS=1 per rank; the (untimed) host generation of each rank's corpus
+    # shares the node's cores instead, set before the generator's OpenMP runtime loads
+    lw = int(os.environ.get("LOCAL_WORLD_SIZE", "1"))
+    if lw > 1:
+        os.environ["OMP_NUM_THREADS"] = str(max(1, (os.cpu_count() or 1) // lw))
     if args.impl == "reference":
         return run_reference(args)
     return run_ours(args)

@@ -290,14 +290,27 @@ static sfs_status refine_hyb(const DevCSR& d, const DevAggr& a, long long rmax, 
   return SFS_OK;
 }
 
+// Host memory the device can store to with the same address (cudaMallocHost under unified addressing).
+static bool host_mapped(const void* p) {
+  cudaPointerAttributes at;
+  if (cudaPointerGetAttributes(&at, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return at.type == cudaMemoryTypeHost && at.devicePointer == p;
+}
+
 // Feature pass for one device CSR; leaves the bitmap in `w` (caller frees) and copies aggregates to `ha`.
 static sfs_status features_device(const DevCSR& d, const sfs_race_opts& o, FeatWork& w, DevAggr* ha_pinned,
                                   cudaStream_t s) {
   void* base = dalloc(feat_work_bytes(d.m, d.n), s);
   if (!base) return fail(SFS_ERR_OOM, "feature workspace");
   feat_work_bind(w, base, d.m, d.n);
-  TRY_CUDA(launch_features(d.rp, d.col, d.m, d.n, d.z, hyb_rmax(d.m, o), w, s));
-  TRY_CUDA(cudaMemcpyAsync(ha_pinned, w.aggr, sizeof(DevAggr), cudaMemcpyDeviceToHost, s));
+  // the last feature kernel writes the aggregates straight into the mapped pinned record (no D2H copy
+  // operation in the stream); unmapped host memory gets a copy
+  const bool mapped = host_mapped(ha_pinned);
+  TRY_CUDA(launch_features(d.rp, d.col, d.m, d.n, d.z, hyb_rmax(d.m, o), w, mapped ? ha_pinned : nullptr, s));
+  if (!mapped) TRY_CUDA(cudaMemcpyAsync(ha_pinned, w.aggr, sizeof(DevAggr), cudaMemcpyDeviceToHost, s));
   return SFS_OK;
 }
 

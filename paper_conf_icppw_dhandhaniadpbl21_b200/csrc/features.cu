@@ -169,55 +169,86 @@ __global__ void k_popcount(const unsigned* __restrict__ bitmap, long long words,
   if ((threadIdx.x & 31) == 0 && c) atomicAdd(&ag->ndiag, c);
 }
 
-// One warp.  j = rmax + 1.  The HYB width rule of Q6 (smallest k >= 1 with R(k) <= rmax, R(k) = #rows
-// longer than k) equals max(1, j-th largest row length); zero rows -> 0.  Lane l owns histogram
-// bins [kHistCap - 128(l+1), kHistCap - 128 l), i.e. lane 0 the longest lengths.
-__global__ void k_hyb_select(long long m, long long j, DevAggr* __restrict__ ag, const unsigned* __restrict__ hist) {
-  const int l = threadIdx.x;
-  if (l == 0) ag->empty_rows = hist[0];
+// One CTA of kSelThreads.  j = rmax + 1.  The HYB width rule of Q6 (smallest k >= 1 with R(k) <= rmax,
+// R(k) = #rows longer than k) equals max(1, j-th largest row length); zero rows -> 0.  Thread t owns
+// histogram bins [kHistCap - 4(t+1), kHistCap - 4t), i.e. thread 0 the longest lengths; a block-wide
+// top-down prefix sum of the per-thread counts locates the bin holding the j-th largest length.
+constexpr int kSelThreads = kHistCap / 4;
+// Thread 0 makes every write to *ag here; it finishes by copying the whole aggregate record into
+// host_out (pinned host memory mapped into the device address space; null = the caller copies).
+__device__ __forceinline__ void publish(const DevAggr* ag, DevAggr* host_out) {
+  if (host_out) *host_out = *ag;
+}
+
+__global__ void __launch_bounds__(kSelThreads) k_hyb_select(long long m, long long j, DevAggr* __restrict__ ag,
+                                                            const unsigned* __restrict__ hist,
+                                                            DevAggr* __restrict__ host_out) {
+  __shared__ long long s_w[kSelThreads / 32];
+  __shared__ long long s_L;
+  const int t = threadIdx.x, l = t & 31, w = t >> 5;
+  if (t == 0) ag->empty_rows = hist[0];
   const long long mx = (long long)ag->max_len;
   const long long bc = (long long)ag->big_cnt, bs = (long long)ag->big_sum;
   if (mx == 0) {
-    if (l == 0) { ag->hyb_k = 0; ag->hyb_coo = 0; }
+    if (t == 0) { ag->hyb_k = 0; ag->hyb_coo = 0; publish(ag, host_out); }
     return;
   }
   if (j <= bc) {  // the order statistic lies beyond the exact histogram: host refines
-    if (l == 0) { ag->hyb_k = -1; ag->hyb_coo = -1; }
+    if (t == 0) { ag->hyb_k = -1; ag->hyb_coo = -1; publish(ag, host_out); }
     return;
   }
-  constexpr int kChunk = kHistCap / 32;
-  const int hi = kHistCap - kChunk * l;  // exclusive
-  const int lo = hi - kChunk;
-  long long mine = 0;
-  for (int b = lo; b < hi; b++) mine += hist[b];
-  long long incl = mine;  // inclusive prefix over lanes 0..l (top-down)
+  const int hi = kHistCap - 4 * t;  // exclusive
+  const int lo = hi - 4;
+  unsigned h[4];
+#pragma unroll
+  for (int q = 0; q < 4; q++) h[q] = hist[lo + q];
+  const long long mine = (long long)h[0] + h[1] + h[2] + h[3];
+  long long incl = mine;  // inclusive prefix over threads 0..t (top-down)
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    long long u = __shfl_up_sync(0xffffffffu, incl, o);
+    const long long u = __shfl_up_sync(0xffffffffu, incl, o);
     if (l >= o) incl += u;
   }
-  const long long above = bc + incl - mine;  // rows longer than any bin of this lane
-  long long L = 0;
-  bool found = false;
+  if (l == 31) s_w[w] = incl;
+  if (t == 0) s_L = 0;  // j exceeds the number of rows
+  __syncthreads();
+  if (w == 0) {
+    long long v = s_w[l], x = v;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const long long u = __shfl_up_sync(0xffffffffu, x, o);
+      if (l >= o) x += u;
+    }
+    s_w[l] = x - v;  // exclusive prefix of the warps before l
+  }
+  __syncthreads();
+  const long long above = bc + s_w[w] + incl - mine;  // rows longer than any bin of this thread
   if (above < j && above + mine >= j) {
     long long cum = above;
-    for (int b = hi - 1; b >= lo; b--) {
-      cum += hist[b];
-      if (cum >= j) { L = b; break; }
+    for (int q = 3; q >= 0; q--) {
+      cum += h[q];
+      if (cum >= j) { s_L = lo + q; break; }
     }
-    found = true;
   }
-  unsigned ballot = __ballot_sync(0xffffffffu, found);
-  if (ballot) L = __shfl_sync(0xffffffffu, L, __ffs(ballot) - 1);
-  else L = 0;  // j exceeds the number of rows
+  __syncthreads();
+  const long long L = s_L;
   const long long K = L < 1 ? 1 : L;
-  long long coo = 0;
-  for (int b = lo; b < hi; b++)
-    if (b > K) coo += (long long)(b - K) * hist[b];
+  unsigned long long coo = 0;
+#pragma unroll
+  for (int q = 0; q < 4; q++)
+    if (lo + q > K) coo += (unsigned long long)(lo + q - K) * h[q];
   coo = warp_sum(coo);
-  if (l == 0) {
-    ag->hyb_k = K;
-    ag->hyb_coo = coo + (bs - K * bc);
+  __syncthreads();
+  if (l == 0) s_w[w] = (long long)coo;
+  __syncthreads();
+  if (w == 0) {
+    unsigned long long c = (unsigned long long)s_w[l];
+    c = warp_sum(c);
+    if (l == 0) {
+      ag->hyb_k = K;
+      ag->hyb_coo = (long long)c + (bs - K * bc);
+      publish(ag, host_out);
+    }
   }
 }
 
@@ -263,14 +294,14 @@ void feat_work_bind(FeatWork& w, void* base, long long m, long long n) {
 }
 
 cudaError_t launch_features(const int* rp, const int* col, long long m, long long n, long long z, long long rmax,
-                            const FeatWork& w, cudaStream_t s) {
+                            const FeatWork& w, DevAggr* host_out, cudaStream_t s) {
   cudaError_t e = cudaMemsetAsync(w.base, 0, w.bytes, s);
   if (e != cudaSuccess) return e;
   k_rowstats<<<grid_for(m, kRowThreads, 4), kRowThreads, 0, s>>>(rp, m, z, w.aggr, w.hist);
   long long tiles = ceil_div(m + z, kNnzTile);
   if (tiles > 0) k_nnzpass<<<(unsigned)tiles, kNnzThreads, 0, s>>>(rp, col, m, n, z, w.aggr, w.bitmap, w.words);
   k_popcount<<<grid_for(w.words, 256, 8), 256, 0, s>>>(w.bitmap, w.words, w.aggr);
-  k_hyb_select<<<1, 32, 0, s>>>(m, rmax + 1, w.aggr, w.hist);
+  k_hyb_select<<<1, kSelThreads, 0, s>>>(m, rmax + 1, w.aggr, w.hist, host_out);
   count_launch(tiles > 0 ? 4 : 3);
   return cudaGetLastError();
 }

@@ -65,7 +65,7 @@ size_t feat_work_bytes(long long m, long long n);
 void feat_work_bind(FeatWork& w, void* base, long long m, long long n);
 // memset + row stats + nnz pass + diag count + HYB select (4 kernels + 1 memset)
 cudaError_t launch_features(const int* rp, const int* col, long long m, long long n, long long z, long long rmax,
-                            const FeatWork& w, cudaStream_t s);
+                            const FeatWork& w, DevAggr* host_out, cudaStream_t s);
 // refine pass of the HYB order statistic: histogram of lengths in [lo, hi] with bin width wdt
 cudaError_t launch_len_hist_range(const int* rp, long long m, long long lo, long long hi, long long wdt,
                                   unsigned* hist, cudaStream_t s);
