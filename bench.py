@@ -326,9 +326,11 @@ def run_ours(args):
         tt = sum(L["t_spmv_us"][f] for L in labs if L["status"][f] == 0) * args.reps
         bb = sum(L["bytes"][f] for L in labs if L["status"][f] == 0) * args.reps
         big = [(L["bytes"][f], L["t_spmv_us"][f]) for L in labs if L["status"][f] == 0 and L["bytes"][f] > 256e6]
+        flops = sum(2.0 * feats[k]["nnz"] for k, L in enumerate(labs) if L["status"][f] == 0) * args.reps
         per_fmt[sfs.FORMAT_NAMES[f]] = {
             "matrices": sum(1 for L in labs if L["status"][f] == 0),
             "spmv_time_s": tt / 1e6, "gbs": (bb / (tt / 1e6) / 1e9) if tt else None,
+            "gflops": (flops / (tt / 1e6) / 1e9) if tt else None,
             "gbs_footprint_gt_2xL2": (sum(b for b, _ in big) / (sum(t for _, t in big) / 1e6) / 1e9) if big else None,
             "labels": sum(1 for L in labs if L["label"] == f),
             "convert_over_csr_spmv": (statistics.median(
