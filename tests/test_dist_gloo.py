@@ -283,7 +283,6 @@ def test_push_runs_deliver_the_ghosts(kind, world):
         assert np.array_equal(xs[k], np.concatenate([x[P.lo], x[P.r0:P.r1], x[P.hi]]))
         runs = sd.push_runs(P, {j: offs[j][k] for j, _, _ in P.send})
         assert sum(e - b for _, b, e, _ in runs) == len(P.send_idx)
-        cover = np.zeros(P.n_local, np.int64)
         for j, b, e, o in runs:
             assert 0 <= b < e <= P.n_local
         nb = sd.push_neighbours(P)
