@@ -290,3 +290,20 @@ def test_push_runs_deliver_the_ghosts(kind, world):
         if kind == "stencil":
             assert len(runs) == len(P.send) <= 2
             assert nb == [j for j in (k - 1, k + 1) if 0 <= j < world]
+
+
+def test_push_struct_marshalling():
+    """sfs_push_t as the binding fills it (host only): counts, runs, flag addresses and epochs; limits of
+    include/sfs.h (SFS_MAX_PUSH runs, SFS_MAX_PEERS flags) are enforced before the C call."""
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    p = sfs.push_struct([(0, 10, 0x1000), (90, 100, 0x2000)], [0x10, 0x14], 7, [0x30], 8, 0x40)
+    assert p.nseg == 2 and (p.seg_begin[1], p.seg_end[1], p.seg_dst[1]) == (90, 100, 0x2000)
+    assert p.nwait == 2 and p.wait_flag[1] == 0x14 and p.wait_value == 7
+    assert p.nsig == 1 and p.sig_flag[0] == 0x30 and p.sig_value == 8 and p.counter == 0x40
+    with pytest.raises(sfs.SfsError):
+        sfs.push_struct([(i, i + 1, 0x1000) for i in range(sfs.MAX_PUSH + 1)], [], 0, [], 1, 0x40)
+    with pytest.raises(sfs.SfsError):
+        sfs.push_struct([], [0x10] * (sfs.MAX_PEERS + 1), 0, [], 1, 0x40)
+    B = sd._PushBuffers(1000, 4, 8)  # x_ext double buffer, flags[world], counter: disjoint, in order
+    assert B.x(0, 1) == 8000 and B.flag(0, 0) == 16000 and B.flag(0, 3) == 16012 and B.counter(0) == 16016
+    assert B.nbytes >= 16020 and B.nbytes % 256 == 0
