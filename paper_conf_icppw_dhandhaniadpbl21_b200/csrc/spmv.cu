@@ -1239,7 +1239,18 @@ template <typename T, bool PUSH>
 cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushParam<PUSH> push) {
   const long long m = A->m;
   const long long blocks_rows = ceil_div(m, dia_rows<T>());  // threads needed at S = 1
-  const int S = split_factor(blocks_rows, A->ndiag, 2 * dia_batch<T>(), 16);
+  int S = split_factor(blocks_rows, A->ndiag, 2 * dia_batch<T>(), 16);
+  // bandwidth-bound fp64: parts of ~12+ diagonals stream faster than one long walk (measured, cold,
+  // tools/micro.py: 128^3 27-point S 1 -> 2: 0.91 -> 0.93 of peak; 1M-row band of 49 diagonals S 2 -> 4:
+  // 0.73 -> 0.80); fp32 keeps the latency rule (its S = 1 is fastest)
+  if (sizeof(T) == 8)
+    while (S < 16 && A->ndiag / (2 * S) >= 12) S <<= 1;
+  static int force_s = -2;  // SFS_DIA_S: A/B override of the diagonal split (1, 2, 4, 8, 16)
+  if (force_s == -2) {
+    const char* e = getenv("SFS_DIA_S");
+    force_s = e ? atoi(e) : -1;
+  }
+  if (force_s == 1 || force_s == 2 || force_s == 4 || force_s == 8 || force_s == 16) S = force_s;
   const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
   const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
   const dim3 gd(grid < 1 ? 1 : grid), bd(kDiaThreads);
