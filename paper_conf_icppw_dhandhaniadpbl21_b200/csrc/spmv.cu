@@ -1158,6 +1158,99 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
   pdl_trigger();
 }
 
+// fp32 DIA: thread = 4 CONSECUTIVE rows, so a diagonal's slab values are one 16-byte vector per thread
+// (the ELL mapping; warp = 128 consecutive rows, 512 contiguous bytes per slab load) and its 4 x values
+// are 4 scalar loads hitting the same lines (L1).  fp32's scalar strided mapping above moves 4 bytes
+// per load instruction; this one moves 16.  S diagonal-parts per row block meet in shared memory.
+template <int S, bool PUSH>
+__global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_f4(const int* __restrict__ offs,
+                                                                const float* __restrict__ dval,
+                                                                const float* __restrict__ x, float* __restrict__ y,
+                                                                long long m, long long n, long long P, int nd,
+                                                                PushParam<PUSH> push) {
+  constexpr int G = kDiaThreads / S;
+  constexpr int kB = 4;  // diagonals per batch
+  __shared__ int s_off[kDiaSmemOffs];
+  __shared__ acc_t s_part[S > 1 ? kDiaThreads * 4 : 1];
+  pdl_wait();
+  pdl_early();
+  const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
+  for (int i = threadIdx.x; i < nsm; i += blockDim.x) s_off[i] = offs[i];
+  __syncthreads();
+  halo_wait<PUSH>(push);
+  bool pushed = false;
+  const int p = threadIdx.x / G, g = threadIdx.x % G;
+  const int Dp = (nd + S - 1) / S;
+  const int d0 = p * Dp, d1 = d0 + Dp < nd ? d0 + Dp : nd;
+  constexpr long long rows_per_blk = (long long)G * 4;
+  const long long nblk = ceil_div(m, rows_per_blk);
+  for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+    const long long r0 = blk * rows_per_blk + 4 * g;  // < P whenever < m (P is a multiple of 32)
+    const bool live = r0 < m;
+    acc_t acc[4] = {0, 0, 0, 0};
+    if (live) {
+      const bool full = r0 + 4 <= m;
+      for (int d = d0; d < d1; d += kB) {
+        const int nb = d1 - d < kB ? d1 - d : kB;
+        int off[kB];
+#pragma unroll
+        for (int u = 0; u < kB; u++) off[u] = u < nb ? (d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u)) : 0;
+        bool all_in = full && nb == kB;
+#pragma unroll
+        for (int u = 0; u < kB; u++) all_in = all_in && r0 + off[u] >= 0 && r0 + off[u] + 3 < n;
+        if (all_in) {
+          float4 v[kB];
+          float xv[kB][4];
+#pragma unroll
+          for (int u = 0; u < kB; u++) v[u] = ld_stream4(dval + (long long)(d + u) * P + r0);
+#pragma unroll
+          for (int u = 0; u < kB; u++) {
+            const float* xp = x + r0 + off[u];
+#pragma unroll
+            for (int q = 0; q < 4; q++) xv[u][q] = ld_x(xp + q);
+          }
+#pragma unroll
+          for (int u = 0; u < kB; u++) {
+            acc[0] += (acc_t)v[u].x * (acc_t)xv[u][0];
+            acc[1] += (acc_t)v[u].y * (acc_t)xv[u][1];
+            acc[2] += (acc_t)v[u].z * (acc_t)xv[u][2];
+            acc[3] += (acc_t)v[u].w * (acc_t)xv[u][3];
+          }
+        } else {
+          for (int u = 0; u < nb; u++) {
+            const float4 v = ld_stream4(dval + (long long)(d + u) * P + r0);
+            const float vv[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+            for (int q = 0; q < 4; q++) {
+              const long long c = r0 + q + off[u];
+              if (r0 + q < m && c >= 0 && c < n) acc[q] += (acc_t)vv[q] * (acc_t)ld_x(x + c);
+            }
+          }
+        }
+      }
+    }
+    if (S > 1) {
+#pragma unroll
+      for (int q = 0; q < 4; q++) s_part[threadIdx.x * 4 + q] = acc[q];
+      __syncthreads();
+      if (p == 0) {
+#pragma unroll
+        for (int pp = 1; pp < S; pp++)
+#pragma unroll
+          for (int q = 0; q < 4; q++) acc[q] += s_part[(pp * G + g) * 4 + q];
+      }
+      __syncthreads();
+    }
+    if (p == 0 && live) {
+#pragma unroll
+      for (int q = 0; q < 4; q++)
+        if (r0 + q < m) store_row<PUSH>(y, r0 + q, (float)acc[q], push, pushed);
+    }
+  }
+  halo_signal<PUSH>(push, pushed);
+  pdl_trigger();
+}
+
 struct MergeWork {
   int2* coords;
   int* crow;
@@ -1235,6 +1328,15 @@ cudaError_t launch_csr_stream(const int* rp, const int* col, const T* val, const
                   push);
 }
 
+bool dia_f4_enabled() {  // SFS_DIA_F4=0: A/B back to the strided fp32 mapping
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SFS_DIA_F4");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
+
 template <typename T, bool PUSH>
 cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushParam<PUSH> push) {
   const long long m = A->m;
@@ -1257,6 +1359,21 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   const int* offs = (const int*)A->ptr[0];
   const T* dv = (const T*)A->ptr[1];
   const int nd = (int)A->ndiag;
+  if constexpr (sizeof(T) == 4) {
+    if (dia_f4_enabled()) {
+      // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
+      const float* xf = (const float*)x;
+      float* yf = (float*)y;
+      const float* dvf = (const float*)dv;
+      switch (S) {
+        case 1: return launch_k(k_spmv_dia_f4<1, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
+        case 2: return launch_k(k_spmv_dia_f4<2, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
+        case 4: return launch_k(k_spmv_dia_f4<4, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
+        case 8: return launch_k(k_spmv_dia_f4<8, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
+        default: return launch_k(k_spmv_dia_f4<16, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
+      }
+    }
+  }
   switch (S) {
     case 1: return launch_k(k_spmv_dia<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
     case 2: return launch_k(k_spmv_dia<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
