@@ -1158,18 +1158,18 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
   pdl_trigger();
 }
 
-// fp32 DIA: thread = 4 CONSECUTIVE rows, so a diagonal's slab values are one 16-byte vector per thread
+// Consecutive-row DIA (fp32): thread = 4 CONSECUTIVE rows, so a diagonal's slab values are one 16-byte vector per thread
 // (the ELL mapping; warp = 128 consecutive rows, 512 contiguous bytes per slab load) and its 4 x values
 // are 4 scalar loads hitting the same lines (L1).  fp32's scalar strided mapping above moves 4 bytes
 // per load instruction; this one moves 16.  S diagonal-parts per row block meet in shared memory.
-template <int S, bool PUSH>
-__global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_f4(const int* __restrict__ offs,
-                                                                const float* __restrict__ dval,
-                                                                const float* __restrict__ x, float* __restrict__ y,
+template <typename T, int S, bool PUSH>
+__global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __restrict__ offs,
+                                                                const T* __restrict__ dval,
+                                                                const T* __restrict__ x, T* __restrict__ y,
                                                                 long long m, long long n, long long P, int nd,
                                                                 PushParam<PUSH> push) {
   constexpr int G = kDiaThreads / S;
-  constexpr int kB = 4;  // diagonals per batch
+  constexpr int kB = sizeof(T) == 4 ? 4 : 2;  // diagonals per batch (register cap)
   __shared__ int s_off[kDiaSmemOffs];
   __shared__ acc_t s_part[S > 1 ? kDiaThreads * 4 : 1];
   pdl_wait();
@@ -1199,31 +1199,28 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_f4(const int* __res
 #pragma unroll
         for (int u = 0; u < kB; u++) all_in = all_in && r0 + off[u] >= 0 && r0 + off[u] + 3 < n;
         if (all_in) {
-          float4 v[kB];
-          float xv[kB][4];
+          Vec4<T> v[kB];
+          T xv[kB][4];
 #pragma unroll
-          for (int u = 0; u < kB; u++) v[u] = ld_stream4(dval + (long long)(d + u) * P + r0);
+          for (int u = 0; u < kB; u++) v[u].load_stream(dval + (long long)(d + u) * P + r0);
 #pragma unroll
           for (int u = 0; u < kB; u++) {
-            const float* xp = x + r0 + off[u];
+            const T* xp = x + r0 + off[u];
 #pragma unroll
             for (int q = 0; q < 4; q++) xv[u][q] = ld_x(xp + q);
           }
 #pragma unroll
-          for (int u = 0; u < kB; u++) {
-            acc[0] += (acc_t)v[u].x * (acc_t)xv[u][0];
-            acc[1] += (acc_t)v[u].y * (acc_t)xv[u][1];
-            acc[2] += (acc_t)v[u].z * (acc_t)xv[u][2];
-            acc[3] += (acc_t)v[u].w * (acc_t)xv[u][3];
-          }
+          for (int u = 0; u < kB; u++)
+#pragma unroll
+            for (int q = 0; q < 4; q++) acc[q] += (acc_t)v[u].v[q] * (acc_t)xv[u][q];
         } else {
           for (int u = 0; u < nb; u++) {
-            const float4 v = ld_stream4(dval + (long long)(d + u) * P + r0);
-            const float vv[4] = {v.x, v.y, v.z, v.w};
+            Vec4<T> v;
+            v.load_stream(dval + (long long)(d + u) * P + r0);
 #pragma unroll
             for (int q = 0; q < 4; q++) {
               const long long c = r0 + q + off[u];
-              if (r0 + q < m && c >= 0 && c < n) acc[q] += (acc_t)vv[q] * (acc_t)ld_x(x + c);
+              if (r0 + q < m && c >= 0 && c < n) acc[q] += (acc_t)v.v[q] * (acc_t)ld_x(x + c);
             }
           }
         }
@@ -1244,7 +1241,7 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_f4(const int* __res
     if (p == 0 && live) {
 #pragma unroll
       for (int q = 0; q < 4; q++)
-        if (r0 + q < m) store_row<PUSH>(y, r0 + q, (float)acc[q], push, pushed);
+        if (r0 + q < m) store_row<PUSH>(y, r0 + q, (T)acc[q], push, pushed);
     }
   }
   halo_signal<PUSH>(push, pushed);
@@ -1328,13 +1325,17 @@ cudaError_t launch_csr_stream(const int* rp, const int* col, const T* val, const
                   push);
 }
 
-bool dia_f4_enabled() {  // SFS_DIA_F4=0: A/B back to the strided fp32 mapping
-  static int v = -1;
-  if (v < 0) {
+// consecutive-row DIA (k_spmv_dia_v4): fp32 by default (SFS_DIA_F4=0 disables), fp64 on request
+// (SFS_DIA_V4_F64=1) -- A/B switches
+bool dia_v4_enabled(size_t elem) {
+  static int f32 = -1, f64 = -1;
+  if (f32 < 0) {
     const char* e = getenv("SFS_DIA_F4");
-    v = (e && e[0] == '0') ? 0 : 1;
+    f32 = (e && e[0] == '0') ? 0 : 1;
+    const char* d = getenv("SFS_DIA_V4_F64");
+    f64 = (d && d[0] == '1') ? 1 : 0;
   }
-  return v == 1;
+  return elem == 4 ? f32 == 1 : f64 == 1;
 }
 
 template <typename T, bool PUSH>
@@ -1359,19 +1360,14 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   const int* offs = (const int*)A->ptr[0];
   const T* dv = (const T*)A->ptr[1];
   const int nd = (int)A->ndiag;
-  if constexpr (sizeof(T) == 4) {
-    if (dia_f4_enabled()) {
-      // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
-      const float* xf = (const float*)x;
-      float* yf = (float*)y;
-      const float* dvf = (const float*)dv;
-      switch (S) {
-        case 1: return launch_k(k_spmv_dia_f4<1, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
-        case 2: return launch_k(k_spmv_dia_f4<2, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
-        case 4: return launch_k(k_spmv_dia_f4<4, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
-        case 8: return launch_k(k_spmv_dia_f4<8, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
-        default: return launch_k(k_spmv_dia_f4<16, PUSH>, gd, bd, s, offs, dvf, xf, yf, m, A->n, A->pitch, nd, push);
-      }
+  if (dia_v4_enabled(sizeof(T))) {
+    // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
+    switch (S) {
+      case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+      case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+      case 4: return launch_k(k_spmv_dia_v4<T, 4, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+      case 8: return launch_k(k_spmv_dia_v4<T, 8, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+      default: return launch_k(k_spmv_dia_v4<T, 16, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
     }
   }
   switch (S) {
