@@ -337,6 +337,15 @@ def run_ours(args):
                 [L["t_convert_us"][f] / L["t_spmv_us"][0] for L in labs
                  if L["status"][f] == 0 and L["status"][0] == 0 and L["t_spmv_us"][0] > 0]) if f else 0.0),
         }
+    try:  # per-format L2-sector rate from the ncu sector counts of the same race (profiles/r01/traffic_corpus200.json)
+        with open(os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json")) as fh:
+            tjall = json.load(fh)
+        for k, v in per_fmt.items():
+            tk = tjall.get(k)
+            if tk and tk.get("l2_sectors_per_launch") and v["spmv_time_s"]:
+                v["l2_gsectors_per_s"] = tk["l2_sectors_per_launch"] * v["matrices"] * args.reps / v["spmv_time_s"] / 1e9
+    except Exception:
+        pass
     dom = max(per_fmt, key=lambda k: per_fmt[k]["spmv_time_s"])
     peaks = {}
     try:
