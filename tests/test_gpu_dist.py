@@ -260,3 +260,34 @@ def test_push_two_processes_share_one_gpu():
     r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-3000:])
     assert r.stdout.count("matches the oracle") == 8, r.stdout[-2000:]
+
+
+@pytest.mark.parametrize("exchange", ["allgather", "halo", "push"])
+def test_bench_rowpart_tool_runs(exchange):
+    """tools/bench_rowpart.py (configs[3] row partition) end to end at a small grid, one rank: every
+    exchange path prints its JSON line."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "tools", "bench_rowpart.py"), "--N", "24", "--iters", "5",
+                        "--warmup", "2", "--exchange", exchange, "--fmt", "DIA"], cwd=root, capture_output=True,
+                       text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    assert d["exchange"] == exchange and d["t_iter_us"] > 0 and d["agg_spmv_gbs"] > 0
+
+
+def test_bench_corpus2000_tool_runs():
+    """tools/bench_corpus2000.py (configs[4]) on its first 6 matrices, one rank: every matrix labelled."""
+    import json
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, os.path.join(root, "tools", "bench_corpus2000.py"), "--limit", "6", "--reps",
+                        "5"], cwd=root, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-2000:]
+    d = json.loads([l for l in r.stdout.splitlines() if l.startswith("{")][-1])
+    assert d["matrices"] == 6 and d["ok"] and d["value"] > 0
