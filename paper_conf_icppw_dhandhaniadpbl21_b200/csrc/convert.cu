@@ -68,23 +68,28 @@ __global__ void __launch_bounds__(kTileThreads) k_csr2coo(const int* __restrict_
 }
 
 // ELL slab (also the ELL part of HYB).  A CTA owns 128 consecutive rows; their CSR segment is
-// contiguous, so it is staged in smem with coalesced loads, then written slot by slot (coalesced).
+// contiguous, so it is staged in shared memory with coalesced loads, then written slot by slot
+// (coalesced).  The staging capacity follows the slab width (128 * K entries, 2048..8192: dynamic
+// shared memory), so rows of up to K entries stay on the staged path; a CTA whose segment is larger
+// still reads its rows from global memory.
 constexpr int kEllRows = 128;
-constexpr int kSegCap = 2048;
+constexpr int kSegCapMin = 2048;
+constexpr int kSegCapMax = 8192;
 
 template <typename T>
 __global__ void __launch_bounds__(kEllRows) k_csr2ell(const int* __restrict__ rp, const int* __restrict__ col,
                                                       const T* __restrict__ val, long long m, long long P, int K,
-                                                      int* __restrict__ ecol, T* __restrict__ eval) {
-  __shared__ int s_col[kSegCap];
-  __shared__ T s_val[kSegCap];
+                                                      int cap, int* __restrict__ ecol, T* __restrict__ eval) {
+  extern __shared__ __align__(16) unsigned char s_seg[];
+  T* s_val = (T*)s_seg;                          // [cap]
+  int* s_col = (int*)(s_seg + sizeof(T) * cap);  // [cap]
   const long long r0 = (long long)blockIdx.x * kEllRows;
   const long long r = r0 + threadIdx.x;
   const long long rend = r0 + kEllRows < m ? r0 + kEllRows : m;
   int seg0 = 0, seg1 = 0, st = 0, len = 0;
   if (r0 < m) { seg0 = rp[r0]; seg1 = rp[rend]; }
   if (r < m) { st = rp[r]; len = rp[r + 1] - st; }
-  const bool staged = (seg1 - seg0) <= kSegCap;
+  const bool staged = (seg1 - seg0) <= cap;
   if (staged) {
     for (int i = threadIdx.x; i < seg1 - seg0; i += blockDim.x) {
       s_col[i] = col[seg0 + i];
@@ -190,10 +195,20 @@ cudaError_t launch_csr2ell(int dtype, const int* rp, const int* col, const void*
                            int* ecol, void* eval, cudaStream_t s) {
   if (K == 0 || P == 0) return cudaSuccess;
   unsigned g = (unsigned)ceil_div(P, kEllRows);
+  long long cap = (long long)kEllRows * K;
+  cap = cap < kSegCapMin ? kSegCapMin : (cap > kSegCapMax ? kSegCapMax : cap);
+  static bool attr = false;  // opt in to > 48 KB of dynamic shared memory once per process
+  if (!attr) {
+    cudaFuncSetAttribute(k_csr2ell<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSegCapMax * 12);
+    cudaFuncSetAttribute(k_csr2ell<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSegCapMax * 8);
+    attr = true;
+  }
   if (dtype == SFS_F64)
-    k_csr2ell<double><<<g, kEllRows, 0, s>>>(rp, col, (const double*)val, m, P, K, ecol, (double*)eval);
+    k_csr2ell<double><<<g, kEllRows, cap * 12, s>>>(rp, col, (const double*)val, m, P, K, (int)cap, ecol,
+                                                    (double*)eval);
   else
-    k_csr2ell<float><<<g, kEllRows, 0, s>>>(rp, col, (const float*)val, m, P, K, ecol, (float*)eval);
+    k_csr2ell<float><<<g, kEllRows, cap * 8, s>>>(rp, col, (const float*)val, m, P, K, (int)cap, ecol,
+                                                  (float*)eval);
   count_launch();
   return cudaGetLastError();
 }
