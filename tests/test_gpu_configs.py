@@ -65,3 +65,23 @@ def test_config4_corpus2000_largest_sample():
     A = sfsgen.generate(sfsgen.corpus_spec(2000, 164))  # 47.0 M nnz, uniform random, fp64
     assert A.nnz > 40_000_000
     _full_check(A, conv=False, ctx="corpus2000[164]")
+
+
+# fp32 DIA at bandwidth-bound sizes takes the TMA-staged kernel (k_spmv_dia_tma: >= 148*2*1024 rows):
+# the configs[3] stencil in fp32, a ragged stencil (343000 rows: partial last 1024-row block) and a
+# ragged 1M-row band, all formats, element by element against the oracle.
+def test_config3_stencil3d27_128_fp32():
+    A = sfsgen.stencil3d27(128, dtype=sfsgen.F32)
+    fo = _full_check(A, formats=(sfs.ELL, sfs.DIA), conv=True, ctx="configs[3] fp32")
+    assert fo["diagonals"] == 27
+
+
+@pytest.mark.parametrize("mk", ["st70", "band"])
+def test_dia_fp32_bandwidth_bound_ragged(mk):
+    if mk == "st70":
+        A = sfsgen.stencil3d27(70, dtype=sfsgen.F32)
+    else:
+        A = sfsgen.generate(sfsgen.make_spec(sfsgen.BAND, seed=12, m=1_000_003, ia=24, pa=0.8, dtype=sfsgen.F32))
+    assert A.m >= 148 * 2 * 1024 and A.m % 1024 != 0
+    fo = _full_check(A, ctx=f"dia fp32 {mk}")
+    assert (fo["admissible_mask"] >> sfs.DIA) & 1
