@@ -1248,131 +1248,6 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
   pdl_trigger();
 }
 
-// TMA-staged DIA (fp32, bandwidth-bound sizes): the slab of a 1024-row block is streamed into a
-// kDtStages-deep shared-memory ring by cp.async.bulk (one 4 KB copy per diagonal, kDtDiags diagonals
-// per stage, mbarrier complete_tx), so the bytes in flight per SM (~5 stages x 16 KB) no longer depend
-// on registers: k_spmv_dia_v4 keeps only 4 x 16 B per thread in flight at 50 % occupancy (ncu: long
-// scoreboard 10.5 of 14 stall cycles per issue, 0.67 of peak on the 128^3 fp32 stencil).  Thread t
-// owns rows r0 + 4t .. +3 of the block (16-byte smem reads); x gathered as in k_spmv_dia_v4.
-constexpr int kDtRows = kDiaThreads * 4;
-constexpr int kDtDiags = 4;
-constexpr int kDtStages = 4;
-constexpr int kDtCtas = 3;
-constexpr int kDtSmem = kDtStages * kDtDiags * kDtRows * 4;
-__device__ __forceinline__ unsigned dt_smem(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
-__device__ __forceinline__ void dt_expect_tx(uint64_t* b, unsigned bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(dt_smem(b)), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void dt_bulk(void* dst, const void* src, unsigned bytes, uint64_t* b) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-               ::"r"(dt_smem(dst)), "l"(src), "r"(bytes), "r"(dt_smem(b)) : "memory");
-}
-__device__ __forceinline__ void dt_wait(uint64_t* b, unsigned parity) {
-  asm volatile(
-      "{\n .reg .pred p;\n W: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra W;\n}\n"
-      ::"r"(dt_smem(b)), "r"(parity) : "memory");
-}
-
-__device__ __forceinline__ void dt_arrive(uint64_t* b) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(dt_smem(b)) : "memory");
-}
-
-// warps 0..7 consume (thread t: rows 4t..4t+3 of the block), warp 8 produces (lane 0 issues the copies);
-// a stage is refilled once all 8 consumer warps arrived on its empty barrier (no CTA-wide barrier per stage)
-__global__ void __launch_bounds__(kDiaThreads + 32, kDtCtas) k_spmv_dia_tma(const int* __restrict__ offs,
-                                                                const float* __restrict__ dval,
-                                                                const float* __restrict__ x, float* __restrict__ y,
-                                                                long long m, long long n, long long P, int nd) {
-  extern __shared__ __align__(128) unsigned char dt_ring[];
-  float* ring = (float*)dt_ring;  // [kDtStages][kDtDiags][kDtRows]
-  __shared__ __align__(8) uint64_t full[kDtStages], empty[kDtStages];
-  __shared__ int s_off[kDiaSmemOffs];
-  pdl_wait();
-  const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
-  for (int i = threadIdx.x; i < nsm; i += blockDim.x) s_off[i] = offs[i];
-  if (threadIdx.x == 0) {
-    for (int i = 0; i < kDtStages; i++) {
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(dt_smem(&full[i])), "r"(1));
-      asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(dt_smem(&empty[i])), "r"(kDiaThreads / 32));
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-  }
-  __syncthreads();
-  const long long nblk = ceil_div(m, (long long)kDtRows);
-  const int nch = (nd + kDtDiags - 1) / kDtDiags;
-  const long long mine = (long long)blockIdx.x < nblk ? (nblk - 1 - blockIdx.x) / gridDim.x + 1 : 0;
-  const long long items = mine * nch;  // (row block, diagonal chunk) pairs of this CTA, chunk-minor
-  if (threadIdx.x >= kDiaThreads) {  // producer warp
-    if (threadIdx.x == kDiaThreads) {
-      for (long long j = 0; j < items; j++) {
-        const int st = (int)(j % kDtStages);
-        if (j >= kDtStages) dt_wait(&empty[st], (unsigned)((j / kDtStages - 1) & 1));
-        const long long b0 = (blockIdx.x + (j / nch) * gridDim.x) * (long long)kDtRows;
-        const long long rb = P - b0 < kDtRows ? P - b0 : kDtRows;  // P is a multiple of 32: 128-byte copies
-        const int d = (int)(j % nch) * kDtDiags, nb = nd - d < kDtDiags ? nd - d : kDtDiags;
-        dt_expect_tx(&full[st], (unsigned)(nb * rb * 4));
-        for (int u = 0; u < nb; u++)
-          dt_bulk(ring + (st * kDtDiags + u) * kDtRows, dval + (long long)(d + u) * P + b0, (unsigned)(rb * 4),
-                  &full[st]);
-      }
-    }
-    pdl_trigger();
-    return;
-  }
-  acc_t acc[4] = {0, 0, 0, 0};
-  for (long long j = 0; j < items; j++) {
-    const int st = (int)(j % kDtStages);
-    const int c = (int)(j % nch);
-    const long long r0 = (blockIdx.x + (j / nch) * gridDim.x) * (long long)kDtRows + 4 * threadIdx.x;
-    const int d = c * kDtDiags, nb = nd - d < kDtDiags ? nd - d : kDtDiags;
-    dt_wait(&full[st], (unsigned)((j / kDtStages) & 1));
-    if (r0 < m) {
-      int off[kDtDiags];
-#pragma unroll
-      for (int u = 0; u < kDtDiags; u++) off[u] = u < nb ? (d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u)) : 0;
-      bool all_in = r0 + 4 <= m && nb == kDtDiags;
-#pragma unroll
-      for (int u = 0; u < kDtDiags; u++) all_in = all_in && r0 + off[u] >= 0 && r0 + off[u] + 3 < n;
-      const float* sv = ring + st * kDtDiags * kDtRows + 4 * threadIdx.x;
-      if (all_in) {
-        float4 v[kDtDiags];
-        float xv[kDtDiags][4];
-#pragma unroll
-        for (int u = 0; u < kDtDiags; u++) v[u] = *(const float4*)(sv + u * kDtRows);
-#pragma unroll
-        for (int u = 0; u < kDtDiags; u++)
-#pragma unroll
-          for (int q = 0; q < 4; q++) xv[u][q] = ld_x(x + r0 + off[u] + q);
-#pragma unroll
-        for (int u = 0; u < kDtDiags; u++) {
-          acc[0] += (acc_t)v[u].x * (acc_t)xv[u][0];
-          acc[1] += (acc_t)v[u].y * (acc_t)xv[u][1];
-          acc[2] += (acc_t)v[u].z * (acc_t)xv[u][2];
-          acc[3] += (acc_t)v[u].w * (acc_t)xv[u][3];
-        }
-      } else {
-        for (int u = 0; u < nb; u++) {
-#pragma unroll
-          for (int q = 0; q < 4; q++) {
-            const long long col = r0 + q + off[u];
-            if (r0 + q < m && col >= 0 && col < n) acc[q] += (acc_t)sv[u * kDtRows + q] * (acc_t)ld_x(x + col);
-          }
-        }
-      }
-    }
-    __syncwarp();  // this warp is done with stage st
-    if ((threadIdx.x & 31) == 0) dt_arrive(&empty[st]);
-    if (c == nch - 1) {
-#pragma unroll
-      for (int q = 0; q < 4; q++) {
-        if (r0 + q < m) y[r0 + q] = (float)acc[q];
-        acc[q] = 0;
-      }
-    }
-  }
-  pdl_trigger();
-}
-
 struct MergeWork {
   int2* coords;
   int* crow;
@@ -1463,18 +1338,6 @@ bool dia_v4_enabled(size_t elem) {
   return elem == 4 ? f32 == 1 : f64 == 1;
 }
 
-// TMA-staged fp32 DIA (k_spmv_dia_tma) for bandwidth-bound sizes (SFS_DIA_TMA=0 disables: A/B switch)
-bool dia_tma_enabled() {
-  static int on = -1;
-  if (on < 0) {
-    const char* e = getenv("SFS_DIA_TMA");
-    on = (e && e[0] == '0') ? 0 : 1;
-    cudaFuncSetAttribute(k_spmv_dia_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, kDtSmem);
-  }
-  return on == 1;
-}
-constexpr long long kDtMinRows = (long long)kSMs * 2 * kDtRows;  // one full wave of row blocks
-
 template <typename T, bool PUSH>
 cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushParam<PUSH> push) {
   const long long m = A->m;
@@ -1497,25 +1360,6 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   const int* offs = (const int*)A->ptr[0];
   const T* dv = (const T*)A->ptr[1];
   const int nd = (int)A->ndiag;
-  if constexpr (!PUSH && sizeof(T) == 4) {
-    if (S == 1 && nd > 0 && m >= kDtMinRows && dia_tma_enabled()) {
-      const long long nb = ceil_div(m, (long long)kDtRows);
-      const int g = (int)(nb < (long long)kSMs * kDtCtas ? nb : (long long)kSMs * kDtCtas);
-      cudaLaunchConfig_t cfg = {};
-      cfg.gridDim = dim3(g);
-      cfg.blockDim = dim3(kDiaThreads + 32);
-      cfg.dynamicSmemBytes = kDtSmem;
-      cfg.stream = s;
-      cudaLaunchAttribute at[1];
-      at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-      at[0].val.programmaticStreamSerializationAllowed = 1;
-      cfg.attrs = at;
-      cfg.numAttrs = pdl_enabled() ? 1 : 0;
-      count_launch();
-      return cudaLaunchKernelEx(&cfg, k_spmv_dia_tma, offs, (const float*)dv, (const float*)x, (float*)y, m, A->n,
-                                (long long)A->pitch, nd);
-    }
-  }
   if (dia_v4_enabled(sizeof(T))) {
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
     switch (S) {
