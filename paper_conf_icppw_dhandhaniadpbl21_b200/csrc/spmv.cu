@@ -1167,7 +1167,7 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
                                                                 const T* __restrict__ dval,
                                                                 const T* __restrict__ x, T* __restrict__ y,
                                                                 long long m, long long n, long long P, int nd,
-                                                                PushParam<PUSH> push) {
+                                                                PushParam<PUSH> push, int pfd) {
   constexpr int G = kDiaThreads / S;
   constexpr int kB = sizeof(T) == 4 ? 4 : 2;  // diagonals per batch (register cap)
   __shared__ int s_off[kDiaSmemOffs];
@@ -1203,6 +1203,14 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
           T xv[kB][4];
 #pragma unroll
           for (int u = 0; u < kB; u++) v[u].load_stream(dval + (long long)(d + u) * P + r0);
+          // slab of the batch pfd batches ahead into L2 (no registers held): more HBM bytes in flight
+          if (pfd > 0) {
+            const int dp = d + pfd * kB;
+#pragma unroll
+            for (int u = 0; u < kB; u++)
+              if (dp + u < d1)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(dval + (long long)(dp + u) * P + r0));
+          }
 #pragma unroll
           for (int u = 0; u < kB; u++) {
             const T* xp = x + r0 + off[u];
@@ -1361,13 +1369,20 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   const T* dv = (const T*)A->ptr[1];
   const int nd = (int)A->ndiag;
   if (dia_v4_enabled(sizeof(T))) {
+    // L2 prefetch of the next batch's slab (SFS_DIA_PF: distance in batches, 0 = off; A/B switch).
+    // 128^3 fp32 stencil cold (tools/ab_dia_pf.sh): off 54.3 us (0.69), 1: 52.2 us (0.71), 2: 53.2, 3: 55.3
+    static int pfd = -1;
+    if (pfd < 0) {
+      const char* e = getenv("SFS_DIA_PF");
+      pfd = e ? atoi(e) : 1;
+    }
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
     switch (S) {
-      case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
-      case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
-      case 4: return launch_k(k_spmv_dia_v4<T, 4, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
-      case 8: return launch_k(k_spmv_dia_v4<T, 8, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
-      default: return launch_k(k_spmv_dia_v4<T, 16, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
+      case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+      case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+      case 4: return launch_k(k_spmv_dia_v4<T, 4, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+      case 8: return launch_k(k_spmv_dia_v4<T, 8, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+      default: return launch_k(k_spmv_dia_v4<T, 16, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
     }
   }
   switch (S) {
