@@ -610,7 +610,7 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
                                               const int* __restrict__ ca, const int* __restrict__ srow,
-                                              long long nwarps, int* head, const unsigned* __restrict__ bm = nullptr) {
+                                              long long nwarps, int* head, const unsigned* __restrict__ bm, int pf) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
   const long long cb = warp * cpw;
@@ -630,6 +630,17 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
   for (long long ch = cb; ch < ce; ch++) {
     const long long k0 = ch * kTChunk;
     const long long k = k0 + l * kTV;
+    // footprints >> L2 (pf): the next chunk's col (1 KB) and val (1 / 2 KB) into L2, one 128-byte line
+    // per lane (L2-resident matrices skip it: there the prefetches only cost issue slots)
+    if (pf && ch + 1 < ce) {
+      constexpr int kColLines = kTChunk * 4 / 128;
+      const long long kn = k0 + kTChunk;
+      const long long e = l < kColLines ? kn + l * 32 : kn + (long long)(l - kColLines) * (128 / (long long)sizeof(T));
+      if (l < kColLines + kTChunk * (int)sizeof(T) / 128 && e < z) {
+        const void* a = l < kColLines ? (const void*)(col + e) : (const void*)(val + e);
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(a));
+      }
+    }
     const int a_lo = BM ? 0 : __ldg(ca + ch), a_hi = BM ? 0 : __ldg(ca + ch + 1);
     unsigned sb = 0;
     if (BM) sb = (__ldg(bm + ch * (kTChunk / 32) + (l >> 2)) >> ((l & 3) * 8)) & 0xFFu;
@@ -760,12 +771,12 @@ __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __res
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
                                                                const int* __restrict__ ca, const int* __restrict__ srow,
-                                                               const unsigned* __restrict__ bm) {
+                                                               const unsigned* __restrict__ bm, int pf) {
   __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (warp < nwarps)
     csr_tile_warp<T, VEC, BM>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps, s_head[BM ? 0 : threadIdx.x >> 5],
-                              bm);
+                              bm, pf);
   else
     pdl_wait();
   pdl_trigger();
@@ -1416,9 +1427,19 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const dim3 grid((unsigned)ceil_div(g.nwarps, tpb / 32));
         // borrowed arrays (e.g. a row block of a larger CSR) may not be 32 B aligned: scalar loads
         const bool vec = ((((uintptr_t)col) | ((uintptr_t)val)) % 32) == 0;
+        // next-chunk L2 prefetch above SFS_TILE_PF_MB of footprint (default 256 = 2 x L2; < 0: never).
+        // Cold, tools/ab_tile_pf.sh: 1M-row band fp64 0.81 -> 0.85 of peak; applied to every matrix the
+        // corpus CSR race got 2.5 % slower (L2-resident matrices), hence the gate.
+        static long long pf_mb = -2;
+        if (pf_mb == -2) {
+          const char* ev = getenv("SFS_TILE_PF_MB");
+          pf_mb = ev ? atoll(ev) : 256;
+        }
+        const long long foot = 4 * (m + 1) + (4 + (long long)sizeof(T)) * z + (long long)sizeof(T) * (A->n + m);
+        const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
         auto go = [&](auto kern) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
-                          (const int*)w.srow, (const unsigned*)w.bm);
+                          (const int*)w.srow, (const unsigned*)w.bm, pf);
         };
         e = launch_k(k_zero_rows<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, y, (const int*)w.srow, g.nwarps, m);
         if (e == cudaSuccess) {
