@@ -111,6 +111,11 @@ typedef struct {
   int64_t hyb_breakeven; /* (4096) */
   int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream; 3 = tile; 4 = tile with row ids from a row-start bitmap (falls back to 3 when a row is empty) */
   int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (0: direct launches with PDL) */
+  const uint32_t *race_mask; /* sfs_label_corpus only, nullable (HOST array of n): matrix i races the
+                                formats formats_mask & race_mask[i]; 0 = features only (no conversion,
+                                no SpMV; label -1, every status SFS_ERR_NOT_RUN) -- the cluster-subset
+                                labelling of P:L134 / P:L167-169 ("benchmark only one matrix from each
+                                cluster").  NULL = every matrix races formats_mask. */
 } sfs_race_opts;
 
 /* Result of racing one matrix. */
@@ -149,7 +154,9 @@ sfs_status sfs_spmv(sfs_format f, sfs_matrix A, const void *x, void *y, void *st
    SpMVs, `reps` timed SpMVs (CUDA events), free; label = argmin (Q14).  feats / labels are host
    arrays of n entries.  A matrix-level error (e.g. INVALID_CSR) is reported in
    labels[i].matrix_status and does not abort the batch; a format-level error (OOM) only marks
-   status[f].  Host-memory matrices are copied to the device inside the call and stay resident
+   status[f].  A launch error or an unreadable timing event of one format marks status[f] =
+   SFS_ERR_CUDA (detail in sfs_last_error) and keeps that format out of the label; the batch goes on.
+   opt->race_mask restricts the race per matrix (featurisation always runs).  Host-memory matrices are copied to the device inside the call and stay resident
    until it returns (callers batch large corpora).  Syncs.  Returns SFS_OK unless an argument is
    invalid or CUDA fails. */
 sfs_status sfs_label_corpus(const sfs_csr *mats, int64_t n, const sfs_race_opts *opt, sfs_features_t *feats,
@@ -266,6 +273,12 @@ sfs_status sfs_cluster_vote(sfs_cluster_model M, const int32_t *labels, int32_t 
 sfs_status sfs_cluster_predict(sfs_cluster_model M, const double *table1, int64_t q, int32_t *cluster, void *stream);
 sfs_status sfs_cluster_describe(sfs_cluster_model M, sfs_cluster_info *out);
 sfs_status sfs_cluster_free(sfs_cluster_model M);
+/* The PCA eigen-step of sfs_cluster_fit on its own (host arrays, host computation, no GPU needed):
+   leading k eigenpairs of the symmetric n x n matrix cov (row-major, 1 <= k <= n <= 64) by Householder
+   tridiagonalisation + implicit QL; eigval descending, basis k x n (row = eigenvector) with each row's
+   largest-magnitude entry (first on ties) positive (reading F3).  INVALID_ARG on bad sizes,
+   UNSUPPORTED if the iteration does not converge. */
+sfs_status sfs_pca_basis(int32_t n, const double *cov, int32_t k, double *basis, double *eigval);
 
 /* Library version string. */
 const char *sfs_version(void);

@@ -65,7 +65,7 @@ class LayoutStruct(ctypes.Structure):
 class RaceOpts(ctypes.Structure):
     _fields_ = [("reps", _I32), ("warmup", _I32), ("formats_mask", _U32), ("cold", _I32), ("max_fill", _D),
                 ("fill_slack", _I64), ("hyb_rel_speed", _D), ("hyb_breakeven", _I64), ("csr_variant", _I32),
-                ("use_graphs", _I32)]
+                ("use_graphs", _I32), ("race_mask", _P)]
 
 
 class LabelStruct(ctypes.Structure):
@@ -112,16 +112,73 @@ def lib():
         L.sfs_last_error.restype = ctypes.c_char_p
         L.sfs_launch_count.restype = _I64
         L.sfs_version.restype = ctypes.c_char_p
+        L.sfs_set_allocator.argtypes = [_ALLOC_T, _FREE_T]
+        L.sfs_set_allocator.restype = None
         for fn in ("sfs_features", "sfs_convert", "sfs_spmv", "sfs_label_corpus", "sfs_matrix_free",
                    "sfs_matrix_describe"):
             getattr(L, fn).restype = _I32
         _lib = L
+        if os.environ.get("SFS_TORCH_ALLOC", "1") != "0":
+            use_torch_allocator(True)
     return _lib
 
 
 EXPORTED = ["sfs_features", "sfs_convert", "sfs_spmv", "sfs_label_corpus", "sfs_matrix_free",
             "sfs_matrix_describe", "sfs_status_string", "sfs_last_error", "sfs_set_allocator",
             "sfs_default_opts", "sfs_spmv_bytes", "sfs_launch_count", "sfs_version"]
+
+
+# ------------------------------------------------------------------ allocator hook (§8(b) ownership)
+# Library-owned buffers (converted matrices, race temporaries, staged inputs) come from torch's caching
+# allocator, so they share one pool with the caller's tensors.  The library frees stream-ordered on the
+# stream it names; torch's allocator reuses a block on the stream it was allocated on, so a free on a
+# different stream first makes the allocation stream wait for the freeing stream (no reuse while the
+# freeing stream's kernels may still read the block).  SFS_TORCH_ALLOC=0 keeps the library's own CUDA
+# stream-ordered pool.
+_ALLOC_T = ctypes.CFUNCTYPE(_P, ctypes.c_size_t, _P)
+_FREE_T = ctypes.CFUNCTYPE(None, _P, _P)
+_alloc_state = {"on": False, "blocks": {}, "cbs": None}
+
+
+def _torch_alloc(nbytes, stream):
+    try:
+        import torch
+        dev = torch.cuda.current_device()
+        p = torch.cuda.caching_allocator_alloc(int(nbytes), dev, stream or 0)
+        _alloc_state["blocks"][p] = (stream or 0, dev)
+        return p
+    except Exception:  # OOM or torch torn down: the library reports SFS_ERR_OOM
+        return None
+
+
+def _torch_free(ptr, stream):
+    try:
+        import torch
+        a_stream, dev = _alloc_state["blocks"].pop(ptr, (stream or 0, None))
+        if (stream or 0) != a_stream:
+            sa = torch.cuda.ExternalStream(a_stream, device=dev) if a_stream else torch.cuda.default_stream(dev)
+            sf = torch.cuda.ExternalStream(stream, device=dev) if stream else torch.cuda.default_stream(dev)
+            sa.wait_stream(sf)
+        torch.cuda.caching_allocator_delete(ptr)
+    except Exception:
+        pass
+
+
+def use_torch_allocator(enable: bool = True):
+    """Route the library's device allocations through torch's caching allocator (sfs_set_allocator)."""
+    L = lib()
+    if enable and not _alloc_state["on"]:
+        cbs = (_ALLOC_T(_torch_alloc), _FREE_T(_torch_free))
+        _alloc_state["cbs"] = cbs  # keep the trampolines alive while the library may call them
+        L.sfs_set_allocator(cbs[0], cbs[1])
+        _alloc_state["on"] = True
+    elif not enable and _alloc_state["on"]:
+        L.sfs_set_allocator(None, None)
+        _alloc_state["on"] = False
+
+
+def torch_allocator_enabled() -> bool:
+    return _alloc_state["on"]
 
 
 def _check(st: int, what: str):
@@ -172,11 +229,28 @@ class Csr:
         return F64 if self.val.dtype == torch.float64 else F32
 
     def struct(self) -> CsrStruct:
+        """The sfs_csr view.  The library stages all four arrays from one `mem` flag, so they must
+        share a placement: all on one CUDA device, or all in PINNED host memory (pageable host memory
+        would silently serialise the copy-stream pipeline of sfs_label_corpus)."""
         import torch
         for t in (self.rp, self.col):
-            assert t.dtype == torch.int32 and t.is_contiguous()
-        assert self.val.dtype in (torch.float32, torch.float64) and self.val.is_contiguous()
-        mem = MEM_DEVICE if self.rp.is_cuda else MEM_HOST
+            if t.dtype != torch.int32 or not t.is_contiguous():
+                raise SfsError(ERR_INVALID_ARG, "rp / col must be contiguous int32")
+        if self.val.dtype not in (torch.float32, torch.float64) or not self.val.is_contiguous():
+            raise SfsError(ERR_INVALID_ARG, "val must be contiguous float32 / float64")
+        ts = [self.rp, self.col, self.val] + ([self.x] if self.x is not None else [])
+        if self.x is not None and (self.x.dtype != self.val.dtype or not self.x.is_contiguous()):
+            raise SfsError(ERR_INVALID_ARG, "x must be contiguous with the dtype of val")
+        if self.rp.is_cuda:
+            if any((not t.is_cuda) or t.device != self.rp.device for t in ts):
+                raise SfsError(ERR_INVALID_ARG, "mixed placement: rp is on a device, another array is not (or on another device)")
+            mem = MEM_DEVICE
+        else:
+            if any(t.is_cuda for t in ts):
+                raise SfsError(ERR_INVALID_ARG, "mixed placement: rp is in host memory, another array is on a device")
+            if any(t.numel() and not t.is_pinned() for t in ts):
+                raise SfsError(ERR_INVALID_ARG, "host-memory CSR must be pinned (torch.Tensor.pin_memory())")
+            mem = MEM_HOST
         return CsrStruct(self.m, self.n, self.nnz, self.rp.data_ptr(), self.col.data_ptr(), self.val.data_ptr(),
                          self.dtype, mem, self.x.data_ptr() if self.x is not None else None)
 
@@ -322,15 +396,29 @@ def ipc_free(addr: int):
     _check(lib().sfs_ipc_free(addr), "sfs_ipc_free")
 
 
-def label_corpus(mats: Sequence[Csr], opts: Optional[RaceOpts] = None, stream=None):
+def label_corpus(mats: Sequence[Csr], opts: Optional[RaceOpts] = None, stream=None, race_mask=None):
     """Features + format race + labels for a batch (sfs_label_corpus).  Returns (features, labels)
-    as lists of dicts."""
+    as lists of dicts.  race_mask: optional per-matrix format masks (0 = features only; SURVEY §8(f)
+    f2), passed as opts.race_mask."""
     n = len(mats)
     arr = (CsrStruct * max(n, 1))(*[m.struct() for m in mats])
     feats = (FeaturesStruct * max(n, 1))()
     labs = (LabelStruct * max(n, 1))()
+    keep = None
+    if race_mask is not None:
+        if len(race_mask) != n:
+            raise SfsError(ERR_INVALID_ARG, "race_mask needs one entry per matrix")
+        o = RaceOpts()
+        if opts is not None:
+            ctypes.pointer(o)[0] = opts
+        else:
+            lib().sfs_default_opts(ctypes.byref(o))
+        keep = (_U32 * max(n, 1))(*[int(v) & 0xFFFFFFFF for v in race_mask])
+        o.race_mask = ctypes.cast(keep, _P)
+        opts = o
     _check(lib().sfs_label_corpus(arr, n, ctypes.byref(opts) if opts else None, feats, labs, _stream_ptr(stream)),
            "sfs_label_corpus")
+    del keep
     return [feats[i].as_dict() for i in range(n)], [labs[i].as_dict() for i in range(n)]
 
 

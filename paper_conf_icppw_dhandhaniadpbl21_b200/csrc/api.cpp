@@ -44,11 +44,11 @@ static sfs_status cuda_fail(cudaError_t e, const char* what) {
 static void* (*g_user_alloc)(size_t, void*) = nullptr;
 static void (*g_user_free)(void*, void*) = nullptr;
 static std::mutex g_pool_mu;
-static cudaMemPool_t g_pools[64] = {};
+static cudaMemPool_t g_pools[kMaxDevices] = {};
 
 static cudaMemPool_t pool_for_current_device() {
   int dev = 0;
-  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return nullptr;
   std::lock_guard<std::mutex> lk(g_pool_mu);
   if (!g_pools[dev]) {
     cudaMemPoolProps props;
@@ -113,6 +113,7 @@ static void defaults(sfs_race_opts* o) {
   o->hyb_breakeven = 4096;
   o->csr_variant = -1;
   o->use_graphs = 0;  // direct PDL launches: measured faster than per-(matrix, format) graphs
+  o->race_mask = nullptr;
 }
 
 // Q6: largest R with  rel * R < m  or  R < breakeven  (the condition is monotone in R).
@@ -257,7 +258,8 @@ static sfs_status refine_hyb(const DevCSR& d, const DevAggr& a, long long rmax, 
   const long long j = rmax + 1;
   long long lo = kHistCap, hi = (long long)a.max_len, above = 0;
   const int nb = 4096;
-  unsigned* dh = (unsigned*)dalloc(sizeof(unsigned) * nb + sizeof(long long), s);
+  Temps tmp(s);  // freed on every return path
+  unsigned* dh = (unsigned*)tmp.get(sizeof(unsigned) * nb + sizeof(long long));
   if (!dh) return fail(SFS_ERR_OOM, "refine");
   std::vector<unsigned> hh(nb);
   while (true) {
@@ -286,7 +288,6 @@ static sfs_status refine_hyb(const DevCSR& d, const DevAggr& a, long long rmax, 
   TRY_CUDA(launch_hyb_coo(d.rp, d.m, *K, dc, s));
   TRY_CUDA(cudaMemcpyAsync(hcoo, dc, sizeof(long long), cudaMemcpyDeviceToHost, s));
   TRY_CUDA(cudaStreamSynchronize(s));
-  dfree(dh, s);
   return SFS_OK;
 }
 
@@ -350,11 +351,19 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
     }
     return p;
   };
-  auto bail = [&](sfs_status st, const char* what) {
+  auto bail = [&](sfs_status st, const std::string& what) {
     for (int i = 0; i < A->n_owned; i++) dfree(A->owned[i], s);
     delete A;
     return fail(st, what);
   };
+  // every CUDA failure releases the partly built handle (no leak of its pool blocks)
+#define BAIL_CUDA(expr)                                                                             \
+  do {                                                                                              \
+    cudaError_t _e = (expr);                                                                        \
+    if (_e != cudaSuccess)                                                                          \
+      return bail(_e == cudaErrorMemoryAllocation ? SFS_ERR_OOM : SFS_ERR_CUDA,                     \
+                  std::string(#expr) + ": " + cudaGetErrorString(_e));                              \
+  } while (0)
   const long long m = d.m, z = d.z, P = A->pitch;
   switch (fmt) {
     case SFS_CSR: {
@@ -363,10 +372,10 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         int* col = (int*)own(sizeof(int) * std::max(z, 1LL));
         void* val = own(sv * std::max(z, 1LL));
         if (!rp || !col || !val) return bail(SFS_ERR_OOM, "csr copy");
-        TRY_CUDA(cudaMemcpyAsync(rp, d.rp, sizeof(int) * (m + 1), cudaMemcpyDeviceToDevice, s));
+        BAIL_CUDA(cudaMemcpyAsync(rp, d.rp, sizeof(int) * (m + 1), cudaMemcpyDeviceToDevice, s));
         if (z) {
-          TRY_CUDA(cudaMemcpyAsync(col, d.col, sizeof(int) * z, cudaMemcpyDeviceToDevice, s));
-          TRY_CUDA(cudaMemcpyAsync(val, d.val, sv * z, cudaMemcpyDeviceToDevice, s));
+          BAIL_CUDA(cudaMemcpyAsync(col, d.col, sizeof(int) * z, cudaMemcpyDeviceToDevice, s));
+          BAIL_CUDA(cudaMemcpyAsync(val, d.val, sv * z, cudaMemcpyDeviceToDevice, s));
         }
         A->ptr[0] = rp; A->ptr[1] = col; A->ptr[2] = val;
       } else {
@@ -376,13 +385,13 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       if (A->variant == 1) {
         A->work = own(csr_merge_work_bytes(m, z, d.dtype));
         if (!A->work) return bail(SFS_ERR_OOM, "csr merge carries");
-        TRY_CUDA(launch_csr_merge_prepare((const int*)A->ptr[0], m, z, A->work, s));
+        BAIL_CUDA(launch_csr_merge_prepare((const int*)A->ptr[0], m, z, A->work, s));
       } else if ((A->variant == 3 || A->variant == 4) && z > 0) {
         if (A->variant == 4 && f.nnz_min < 1) A->variant = 3;  // the row-start bitmap needs every row non-empty
         const int bitmap = A->variant == 4;
         A->work = own(csr_tile_work_bytes(m, z, bitmap));
         if (!A->work) return bail(SFS_ERR_OOM, "csr tile partition");
-        TRY_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, bitmap, s));
+        BAIL_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, bitmap, s));
       }
       break;
     }
@@ -391,7 +400,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       int* c = (int*)own(sizeof(int) * std::max(z, 1LL));
       void* v = own(sv * std::max(z, 1LL));
       if (!r || !c || !v) return bail(SFS_ERR_OOM, "coo");
-      TRY_CUDA(launch_csr2coo(d.dtype, d.rp, d.col, d.val, m, z, r, c, v, s));
+      BAIL_CUDA(launch_csr2coo(d.dtype, d.rp, d.col, d.val, m, z, r, c, v, s));
       A->ptr[0] = r; A->ptr[1] = c; A->ptr[2] = v;
       break;
     }
@@ -401,7 +410,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       int* ec = (int*)own(sizeof(int) * std::max(K * P, 1LL));
       void* ev = own(sv * std::max(K * P, 1LL));
       if (!ec || !ev) return bail(SFS_ERR_OOM, "ell");
-      TRY_CUDA(launch_csr2ell(d.dtype, d.rp, d.col, d.val, m, P, (int)K, ec, ev, s));
+      BAIL_CUDA(launch_csr2ell(d.dtype, d.rp, d.col, d.val, m, P, (int)K, ec, ev, s));
       A->ptr[0] = ec; A->ptr[1] = ev;
       A->width = K;
       break;
@@ -414,7 +423,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       int* cc = (int*)own(sizeof(int) * std::max(nc, 1LL));
       void* cv = own(sv * std::max(nc, 1LL));
       if (!ec || !ev || !cr || !cc || !cv) return bail(SFS_ERR_OOM, "hyb");
-      TRY_CUDA(launch_csr2ell(d.dtype, d.rp, d.col, d.val, m, P, (int)K, ec, ev, s));
+      BAIL_CUDA(launch_csr2ell(d.dtype, d.rp, d.col, d.val, m, P, (int)K, ec, ev, s));
       // rows overflowing by <= 32 (64 below 2^20 nnz): keep the per-row overflow offsets for the one-launch SpMV
       A->variant = hyb_rowwise(f.nnz_max, K, nc, z);
       if (nc > 0) {
@@ -422,8 +431,8 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         int* ovf = A->variant ? (int*)own(sizeof(int) * (m + 1)) : (int*)t.get(sizeof(int) * (m + 1));
         void* work = t.get(scan_work_bytes(m));
         if (!ovf || !work) return bail(SFS_ERR_OOM, "hyb scan");
-        TRY_CUDA(launch_overflow_scan(d.rp, m, (int)K, ovf, work, s));
-        TRY_CUDA(launch_hyb_coo_part(d.dtype, d.rp, d.col, d.val, m, z, (int)K, ovf, cr, cc, cv, s));
+        BAIL_CUDA(launch_overflow_scan(d.rp, m, (int)K, ovf, work, s));
+        BAIL_CUDA(launch_hyb_coo_part(d.dtype, d.rp, d.col, d.val, m, z, (int)K, ovf, cr, cc, cv, s));
         if (A->variant) A->ptr[5] = ovf;
       }
       A->ptr[0] = ec; A->ptr[1] = ev; A->ptr[2] = cr; A->ptr[3] = cc; A->ptr[4] = cv;
@@ -442,12 +451,12 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         int* wp = (int*)t.get(sizeof(int) * (fw.words + 1));
         void* work = t.get(scan_work_bytes(fw.words));
         if (!wp || !work) return bail(SFS_ERR_OOM, "dia scan");
-        TRY_CUDA(launch_popc_scan(fw.bitmap, fw.words, wp, work, s));
-        TRY_CUDA(launch_dia_offsets(fw.bitmap, fw.words, wp, m, offs, s));
+        BAIL_CUDA(launch_popc_scan(fw.bitmap, fw.words, wp, work, s));
+        BAIL_CUDA(launch_dia_offsets(fw.bitmap, fw.words, wp, m, offs, s));
         if (nd > 0) {
-          TRY_CUDA(cudaMemsetAsync(dv, 0, sv * nd * P, s));
+          BAIL_CUDA(cudaMemsetAsync(dv, 0, sv * nd * P, s));
           count_launch();
-          TRY_CUDA(launch_csr2dia(d.dtype, d.rp, d.col, d.val, m, P, fw.bitmap, wp, dv, s));
+          BAIL_CUDA(launch_csr2dia(d.dtype, d.rp, d.col, d.val, m, P, fw.bitmap, wp, dv, s));
         }
       }
       A->ptr[0] = offs; A->ptr[1] = dv;
@@ -457,6 +466,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
     default:
       return bail(SFS_ERR_INVALID_ARG, "bad format");
   }
+#undef BAIL_CUDA
   *out = A;
   return SFS_OK;
 }
@@ -551,7 +561,10 @@ sfs_status sfs_features(const sfs_csr* A, const sfs_race_opts* opt, sfs_features
   DevCSR d;
   if ((st = stage(A, d, s, false)) != SFS_OK) { unstage(d, s); return st; }
   DevAggr* ha = nullptr;
-  TRY_CUDA(cudaMallocHost(&ha, sizeof(DevAggr)));
+  if (cudaError_t e = cudaMallocHost(&ha, sizeof(DevAggr)); e != cudaSuccess) {
+    unstage(d, s);
+    return cuda_fail(e, "pinned aggregate record");
+  }
   FeatWork w;
   st = features_device(d, o, w, ha, s);
   if (st == SFS_OK) {
@@ -576,7 +589,10 @@ sfs_status sfs_convert(const sfs_csr* A, sfs_format f, const sfs_race_opts* opt,
   DevCSR d;
   if ((st = stage(A, d, s, false)) != SFS_OK) { unstage(d, s); return st; }
   DevAggr* ha = nullptr;
-  TRY_CUDA(cudaMallocHost(&ha, sizeof(DevAggr)));
+  if (cudaError_t e = cudaMallocHost(&ha, sizeof(DevAggr)); e != cudaSuccess) {
+    unstage(d, s);
+    return cuda_fail(e, "pinned aggregate record");
+  }
   FeatWork w;
   sfs_features_t F;
   st = features_device(d, o, w, ha, s);
@@ -654,9 +670,14 @@ sfs_status sfs_ipc_alloc(size_t bytes, void** ptr, uint8_t handle[64]) {
   if (!ptr || !handle || bytes == 0) return fail(SFS_ERR_INVALID_ARG, "null argument / zero size");
   static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
   TRY_CUDA(cudaMalloc(ptr, bytes));
-  TRY_CUDA(cudaMemset(*ptr, 0, bytes));
   cudaIpcMemHandle_t h;
-  TRY_CUDA(cudaIpcGetMemHandle(&h, *ptr));
+  cudaError_t e = cudaMemset(*ptr, 0, bytes);
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(&h, *ptr);
+  if (e != cudaSuccess) {
+    cudaFree(*ptr);
+    *ptr = nullptr;
+    return cuda_fail(e, "sfs_ipc_alloc");
+  }
   memcpy(handle, &h, 64);
   return SFS_OK;
 }
@@ -711,32 +732,67 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   if (opt) o = *opt;
   if (o.reps < 1 || o.warmup < 0) return fail(SFS_ERR_INVALID_ARG, "reps >= 1, warmup >= 0");
   cudaStream_t s = (cudaStream_t)stream;
-  cudaStream_t cap = nullptr;  // capture-only stream (records graphs, executes nothing)
-  TRY_CUDA(cudaStreamCreateWithFlags(&cap, cudaStreamNonBlocking));
-  cudaStream_t up = nullptr;  // graph uploads (SFS_GRAPH_UPLOAD=0 disables)
-  {
-    const char* eu = getenv("SFS_GRAPH_UPLOAD");
-    if (!(eu && eu[0] == '0')) TRY_CUDA(cudaStreamCreateWithFlags(&up, cudaStreamNonBlocking));
-  }
   EventPool ev;
   std::vector<DevCSR> d(n);
   std::vector<FeatWork> w(n);
   std::vector<sfs_status> mst(n, SFS_OK);
   std::vector<cudaEvent_t> fe0(n, nullptr), fe1(n, nullptr), ce(n, nullptr);
-  DevAggr* ha = nullptr;
-  TRY_CUDA(cudaMallocHost(&ha, sizeof(DevAggr) * std::max<int64_t>(n, 1)));
+  struct Timed {
+    int64_t i;
+    int f;
+    cudaEvent_t c0, c1, t0, t1;
+    std::vector<cudaEvent_t> cold;
+  };
+  std::vector<Timed> timed;
+  std::vector<cudaGraphExec_t> execs;
+  std::vector<cudaGraph_t> graphs;
+  // Everything the call owns is released by this guard on every return path (streams, the pinned
+  // aggregate records, graphs, staged inputs, feature workspaces, the L2 flush buffer).
+  struct Owned {
+    cudaStream_t s = nullptr, cap = nullptr, up = nullptr, cs = nullptr;
+    DevAggr* ha = nullptr;
+    void* flush = nullptr;
+    std::vector<DevCSR>* d = nullptr;
+    std::vector<FeatWork>* w = nullptr;
+    std::vector<cudaGraphExec_t>* execs = nullptr;
+    std::vector<cudaGraph_t>* graphs = nullptr;
+    ~Owned() {
+      for (auto ge : *execs) cudaGraphExecDestroy(ge);
+      for (auto g : *graphs) cudaGraphDestroy(g);
+      for (auto& x : *w) dfree(x.base, s);
+      for (auto& x : *d) unstage(x, s);
+      dfree(flush, s);
+      if (cap) cudaStreamDestroy(cap);
+      if (up) cudaStreamDestroy(up);
+      if (cs) cudaStreamDestroy(cs);
+      if (ha) cudaFreeHost(ha);
+    }
+  } own;
+  own.s = s;
+  own.d = &d;
+  own.w = &w;
+  own.execs = &execs;
+  own.graphs = &graphs;
+  TRY_CUDA(cudaStreamCreateWithFlags(&own.cap, cudaStreamNonBlocking));  // capture-only (records graphs)
+  {
+    const char* eu = getenv("SFS_GRAPH_UPLOAD");  // graph uploads on a side stream (0 disables)
+    if (!(eu && eu[0] == '0')) TRY_CUDA(cudaStreamCreateWithFlags(&own.up, cudaStreamNonBlocking));
+  }
+  TRY_CUDA(cudaMallocHost(&own.ha, sizeof(DevAggr) * std::max<int64_t>(n, 1)));
+  cudaStream_t cap = own.cap, up = own.up;
+  DevAggr* ha = own.ha;
   for (int64_t i = 0; i < n; i++) {
     memset(&labels[i], 0, sizeof(sfs_label_t));
     memset(&feats[i], 0, sizeof(sfs_features_t));
     labels[i].label = -1;
     for (int f = 0; f < SFS_NFMT; f++) labels[i].status[f] = SFS_ERR_NOT_RUN;
   }
-  cudaStream_t cs = nullptr;  // H2D copy stream for host-memory inputs
   for (int64_t i = 0; i < n; i++)
-    if (mats[i].mem == SFS_MEM_HOST) {
-      TRY_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    if (mats[i].mem == SFS_MEM_HOST) {  // H2D copy stream for host-memory inputs
+      TRY_CUDA(cudaStreamCreateWithFlags(&own.cs, cudaStreamNonBlocking));
       break;
     }
+  cudaStream_t cs = own.cs;
   // Chunks.  A device-resident corpus is one chunk: every feature pass, one synchronisation (the host
   // needs the features to enqueue the race), then the whole race enqueued.  Host-memory inputs come in
   // chunks of 1, 2, 4, ... matrices: the H2D copies of chunk c+1 (copy stream) run during the race of
@@ -776,33 +832,19 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
   using clk = std::chrono::steady_clock;
   const bool prof = getenv("SFS_PROFILE") != nullptr;
   double t_graph = 0, t_inst = 0, t_conv = 0, t_warm = 0, t_sync = 0;
-  struct Timed {
-    int64_t i;
-    int f;
-    cudaEvent_t c0, c1, t0, t1;
-    std::vector<cudaEvent_t> cold;
-  };
-  std::vector<Timed> timed;
-  std::vector<cudaGraphExec_t> execs;
-  std::vector<cudaGraph_t> graphs;
-  void* flush = nullptr;
   size_t flush_bytes = 0;
-  auto cleanup = [&]() {
-    for (auto ge : execs) cudaGraphExecDestroy(ge);
-    for (auto g : graphs) cudaGraphDestroy(g);
-    cudaStreamDestroy(cap);
-    if (up) cudaStreamDestroy(up);
-    if (cs) cudaStreamDestroy(cs);
-    cudaFreeHost(ha);
-  };
   if (o.cold && n > 0) {
     int dev = 0, l2 = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, dev);
     flush_bytes = (size_t)std::max(l2, 1 << 20) * 2;
-    flush = dalloc(flush_bytes, s);
+    own.flush = dalloc(flush_bytes, s);
   }
-  // the race of one matrix: every admissible format converted, warmed up and timed; nothing synchronises
+  void* flush = own.flush;
+  // The race of one matrix: every format of its race set converted, warmed up and timed; nothing
+  // synchronises.  The race set is formats_mask & race_mask[i] (a matrix with an
+  // empty set is featurised only -- no conversion, no SpMV).  A launch error of any SpMV of a format
+  // marks that format SFS_ERR_CUDA and keeps it out of the label (no silent near-zero time).
   auto race_one = [&](int64_t i) {
     sfs_label_t& L = labels[i];
     if (mst[i] != SFS_OK) {
@@ -813,6 +855,9 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     L.admissible_mask = F.admissible_mask;
     L.csr_variant = F.csr_variant;
     const DevCSR& D = d[i];
+    const uint32_t race_set = o.formats_mask & (o.race_mask ? o.race_mask[i] : 0x1Fu);
+    for (int f = 0; f < SFS_NFMT; f++) L.bytes[f] = sfs_spmv_bytes(&F, (sfs_format)f, (sfs_dtype)D.dtype);
+    if (!(race_set & 0x1Fu)) return;  // features only
     const size_t sv = vbytes(D.dtype);
     void* y = dalloc(sv * D.m, s);
     void* xo = nullptr;
@@ -829,8 +874,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
       return;
     }
     for (int f = 0; f < SFS_NFMT; f++) {
-      L.bytes[f] = sfs_spmv_bytes(&F, (sfs_format)f, (sfs_dtype)D.dtype);
-      if (!(o.formats_mask & (1u << f))) { L.status[f] = SFS_ERR_NOT_RUN; continue; }
+      if (!(race_set & (1u << f))) { L.status[f] = SFS_ERR_NOT_RUN; continue; }
       if (!(F.admissible_mask & (1u << f))) { L.status[f] = SFS_ERR_INADMISSIBLE; continue; }
       Timed T;
       T.i = i;
@@ -845,16 +889,20 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
       const auto tc1 = clk::now();
       t_conv += std::chrono::duration<double>(tc1 - tc0).count();
       if (st != SFS_OK) { L.status[f] = st; continue; }
-      for (int r = 0; r < o.warmup; r++) launch_spmv(A, x, y, s);
+      cudaError_t le = cudaSuccess;  // first launch error of this (matrix, format)
+      auto chk = [&](cudaError_t e) {
+        if (le == cudaSuccess && e != cudaSuccess) le = e;
+      };
+      for (int r = 0; r < o.warmup; r++) chk(launch_spmv(A, x, y, s));
       t_warm += std::chrono::duration<double>(clk::now() - tc1).count();
       const int kpc = spmv_kernels_per_call(A);
       if (o.cold) {
         for (int r = 0; r < o.reps; r++) {
-          if (flush) launch_l2_flush(flush, flush_bytes, s);
+          if (flush) chk(launch_l2_flush(flush, flush_bytes, s));
           cudaEvent_t a = ev.get(), b = ev.get();
-          cudaEventRecord(a, s);
-          launch_spmv(A, x, y, s);
-          cudaEventRecord(b, s);
+          chk(cudaEventRecord(a, s));
+          chk(launch_spmv(A, x, y, s));
+          chk(cudaEventRecord(b, s));
           T.cold.push_back(a);
           T.cold.push_back(b);
         }
@@ -865,8 +913,8 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
         const auto tg0 = clk::now();
         bool ok = cudaStreamBeginCapture(cap, cudaStreamCaptureModeThreadLocal) == cudaSuccess;
         if (ok) {
-          for (int r = 0; r < o.reps; r++) launch_spmv(A, x, y, cap);
-          ok = cudaStreamEndCapture(cap, &g) == cudaSuccess;
+          for (int r = 0; r < o.reps; r++) ok = launch_spmv(A, x, y, cap) == cudaSuccess && ok;
+          ok = cudaStreamEndCapture(cap, &g) == cudaSuccess && ok;
         }
         g_launches.store(before);
         const auto ti0 = clk::now();
@@ -880,28 +928,34 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
         }
         t_inst += std::chrono::duration<double>(clk::now() - ti0).count();
         t_graph += std::chrono::duration<double>(clk::now() - tg0).count();
+        if (ge) execs.push_back(ge);
+        if (g) graphs.push_back(g);
         T.t0 = ev.get();
         T.t1 = ev.get();
-        cudaEventRecord(T.t0, s);
+        chk(cudaEventRecord(T.t0, s));
         if (ok) {
-          cudaGraphLaunch(ge, s);
+          chk(cudaGraphLaunch(ge, s));
           count_launch((int64_t)o.reps * kpc);
-          execs.push_back(ge);
-          graphs.push_back(g);
         } else {
-          cudaGetLastError();
-          if (g) cudaGraphDestroy(g);
-          for (int r = 0; r < o.reps; r++) launch_spmv(A, x, y, s);
+          cudaGetLastError();  // a failed capture falls back to direct launches
+          for (int r = 0; r < o.reps; r++) chk(launch_spmv(A, x, y, s));
         }
-        cudaEventRecord(T.t1, s);
+        chk(cudaEventRecord(T.t1, s));
       } else {
         T.t0 = ev.get();
         T.t1 = ev.get();
-        cudaEventRecord(T.t0, s);
-        for (int r = 0; r < o.reps; r++) launch_spmv(A, x, y, s);
-        cudaEventRecord(T.t1, s);
+        chk(cudaEventRecord(T.t0, s));
+        for (int r = 0; r < o.reps; r++) chk(launch_spmv(A, x, y, s));
+        chk(cudaEventRecord(T.t1, s));
       }
       matrix_free(A);
+      if (le != cudaSuccess) {
+        cudaGetLastError();
+        set_error(std::string("spmv launch (") + std::to_string(i) + ", " + std::to_string(f) +
+                  "): " + cudaGetErrorString(le));
+        L.status[f] = le == cudaErrorMemoryAllocation ? SFS_ERR_OOM : SFS_ERR_CUDA;
+        continue;
+      }
       L.status[f] = SFS_OK;
       timed.push_back(std::move(T));
     }
@@ -918,10 +972,7 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     const auto ts0 = clk::now();
     e = cudaStreamSynchronize(s);  // this chunk's features (and the previous chunk's race) are done
     t_sync += std::chrono::duration<double>(clk::now() - ts0).count();
-    if (e != cudaSuccess) {
-      cleanup();
-      return cuda_fail(e, c == 0 ? "feature phase" : "race");
-    }
+    if (e != cudaSuccess) return cuda_fail(e, c == 0 ? "feature phase" : "race");
     for (int64_t i = cb[c]; i < cb[c + 1]; i++) {
       if (mst[i] == SFS_OK) mst[i] = features_finish(d[i], o, ha[i], &feats[i], s);
       if (mst[i] == SFS_OK) labels[i].t_features_us = elapsed_us(fe0[i], fe1[i]);
@@ -936,7 +987,6 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
     }
     if (c + 1 < nchunks) features_chunk(c + 1);
   }
-  if (flush) dfree(flush, s);
   const auto t_enq = clk::now();
   e = cudaStreamSynchronize(s);
   if (prof) {
@@ -948,18 +998,28 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
             1e3 * t_warm, 1e3 * (t_graph - t_inst), 1e3 * t_inst, 1e3 * t_sync,
             1e3 * std::chrono::duration<double>(t_end - t_enq).count());
   }
-  cleanup();
   if (e != cudaSuccess) return cuda_fail(e, "race");
   for (auto& T : timed) {
     sfs_label_t& L = labels[T.i];
     L.t_convert_us[T.f] = T.f == SFS_CSR ? 0.f : elapsed_us(T.c0, T.c1);
+    double t = 0;
     if (o.cold) {
-      double sum = 0;
-      for (size_t k = 0; k + 1 < T.cold.size(); k += 2) sum += elapsed_us(T.cold[k], T.cold[k + 1]);
-      L.t_spmv_us[T.f] = (float)(sum / o.reps);
+      for (size_t k = 0; k + 1 < T.cold.size(); k += 2) {
+        const float u = elapsed_us(T.cold[k], T.cold[k + 1]);
+        t = (u < 0 || t < 0) ? -1.0 : t + u;
+      }
+      if (t >= 0) t /= o.reps;
     } else {
-      L.t_spmv_us[T.f] = elapsed_us(T.t0, T.t1) / (float)o.reps;
+      const float u = elapsed_us(T.t0, T.t1);
+      t = u < 0 ? -1.0 : (double)u / o.reps;
     }
+    if (!(t >= 0)) {  // an event that cannot be read is a failed format, not a time
+      L.status[T.f] = SFS_ERR_CUDA;
+      L.t_spmv_us[T.f] = 0.f;
+      set_error("race: unreadable timing event");
+      continue;
+    }
+    L.t_spmv_us[T.f] = (float)t;
   }
   // label: argmin over formats that ran, ties to the lowest id (Q14)
   for (int64_t i = 0; i < n; i++) {

@@ -3,8 +3,8 @@
 // to [0, 1] -> PCA(8) -> K-Means -> majority vote of the benchmarked members per cluster -> nearest
 // centroid for new matrices.  Readings F1–F7: DESIGN.md.
 //
-// Work split: the per-element transform (glibc log1p / sqrt) and the 21x21 Jacobi eigensolver run on
-// the host; everything that scales with the corpus (min/max, covariance, projection, every K-Means
+// Work split: the per-element transform (glibc log1p / sqrt) and the 21x21 symmetric eigensolver
+// (eigen.cpp: Householder + implicit QL) run on the host; everything that scales with the corpus (min/max, covariance, projection, every K-Means
 // assignment and update, votes, prediction) runs in the kernels below.  All device arithmetic uses
 // explicitly rounded intrinsics (__dadd_rn / __dmul_rn / __dsub_rn / __ddiv_rn: never contracted into
 // FMAs) in the fixed orders of the definitions, so results are reproducible bit for bit.
@@ -161,70 +161,6 @@ __global__ void k_vote(const int* __restrict__ assign, const int* __restrict__ l
   out[c] = best >= 0 ? best : gl;
 }
 
-// F3 host part: cyclic Jacobi of the 21x21 covariance, eigenvectors sorted by descending eigenvalue
-// (stable) with the largest-magnitude entry made positive; basis is k x 21.
-void jacobi_basis(const double* Cin, int k, double* basis, double* eigval) {
-  double C[kF * kF], V[kF * kF];
-  memcpy(C, Cin, sizeof(C));
-  for (int i = 0; i < kF * kF; i++) V[i] = 0.0;
-  for (int a = 0; a < kF; a++) V[a * kF + a] = 1.0;
-  for (int sweep = 0; sweep < 64; sweep++) {
-    bool rotated = false;
-    for (int p = 0; p < kF; p++)
-      for (int q = p + 1; q < kF; q++) {
-        const double apq = C[p * kF + q];
-        if (apq == 0.0) continue;
-        const double app = C[p * kF + p], aqq = C[q * kF + q];
-        const double theta = (aqq - app) / (2.0 * apq);
-        double t = 1.0 / (fabs(theta) + sqrt(theta * theta + 1.0));
-        if (theta < 0.0) t = -t;
-        const double c = 1.0 / sqrt(t * t + 1.0), s = t * c;
-        if (s == 0.0) {
-          C[p * kF + q] = C[q * kF + p] = 0.0;
-          continue;
-        }
-        rotated = true;
-        for (int r = 0; r < kF; r++) {
-          const double crp = C[r * kF + p], crq = C[r * kF + q];
-          C[r * kF + p] = c * crp - s * crq;
-          C[r * kF + q] = s * crp + c * crq;
-        }
-        for (int r = 0; r < kF; r++) {
-          const double cpr = C[p * kF + r], cqr = C[q * kF + r];
-          C[p * kF + r] = c * cpr - s * cqr;
-          C[q * kF + r] = s * cpr + c * cqr;
-        }
-        C[p * kF + q] = C[q * kF + p] = 0.0;
-        for (int r = 0; r < kF; r++) {
-          const double vrp = V[r * kF + p], vrq = V[r * kF + q];
-          V[r * kF + p] = c * vrp - s * vrq;
-          V[r * kF + q] = s * vrp + c * vrq;
-        }
-      }
-    if (!rotated) break;
-  }
-  int order[kF];
-  for (int a = 0; a < kF; a++) order[a] = a;
-  for (int a = 1; a < kF; a++) {
-    const int o = order[a];
-    int b = a - 1;
-    while (b >= 0 && C[order[b] * kF + order[b]] < C[o * kF + o]) {
-      order[b + 1] = order[b];
-      b--;
-    }
-    order[b + 1] = o;
-  }
-  for (int c = 0; c < k; c++) {
-    const int col = order[c];
-    eigval[c] = C[col * kF + col];
-    int big = 0;
-    for (int r = 1; r < kF; r++)
-      if (fabs(V[r * kF + col]) > fabs(V[big * kF + col])) big = r;
-    const double sg = V[big * kF + col] < 0.0 ? -1.0 : 1.0;
-    for (int r = 0; r < kF; r++) basis[c * kF + r] = sg * V[r * kF + col];
-  }
-}
-
 void transform_host(const double* raw, long long n, std::vector<double>& out) {
   out.resize((size_t)n * kF);
   for (long long i = 0; i < n; i++)
@@ -282,7 +218,8 @@ cudaError_t cluster_fit(const double* raw, long long n, const int* init_idx, int
   if ((e = cudaStreamSynchronize(s)) != cudaSuccess) return e;
   M->basis.resize((size_t)k * kF);
   M->eigval.resize(k);
-  jacobi_basis(C, k, M->basis.data(), M->eigval.data());
+  // F3: Householder tridiagonalisation + implicit QL (eigen.cpp; independent of the oracle's Jacobi)
+  if (!sym_eigen_basis(kF, C, k, M->basis.data(), M->eigval.data())) return cudaErrorUnknown;
   if ((e = cudaMemcpyAsync(dbasis, M->basis.data(), sizeof(double) * k * kF, cudaMemcpyHostToDevice, s)) != cudaSuccess)
     return e;
   k_project<<<blocks_for(n * k, 256), 256, 0, s>>>(dX, n, dmean, dbasis, k, dY);

@@ -8,6 +8,8 @@
 //   HYB : ELL slab of width K_hyb + COO part (entries j >= K_hyb of each row, (r, j) order).
 //   DIA : offsets ascending + slab val[d*P + r] (+0 where the entry is absent).
 #include "common.cuh"
+#include <mutex>
+
 #include "internal.h"
 
 namespace sfs {
@@ -197,12 +199,14 @@ cudaError_t launch_csr2ell(int dtype, const int* rp, const int* col, const void*
   unsigned g = (unsigned)ceil_div(P, kEllRows);
   long long cap = (long long)kEllRows * K;
   cap = cap < kSegCapMin ? kSegCapMin : (cap > kSegCapMax ? kSegCapMax : cap);
-  static bool attr = false;  // opt in to > 48 KB of dynamic shared memory once per process
-  if (!attr) {
+  // opt in to > 48 KB of dynamic shared memory: a function attribute is per device, so once per device
+  static std::once_flag attr_once[kMaxDevices];
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+  std::call_once(attr_once[dev], [] {
     cudaFuncSetAttribute(k_csr2ell<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSegCapMax * 12);
     cudaFuncSetAttribute(k_csr2ell<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSegCapMax * 8);
-    attr = true;
-  }
+  });
   if (dtype == SFS_F64)
     k_csr2ell<double><<<g, kEllRows, cap * 12, s>>>(rp, col, (const double*)val, m, P, K, (int)cap, ecol,
                                                     (double*)eval);

@@ -25,6 +25,7 @@ void set_error(const std::string& msg);
   } while (0)
 
 // ---------------------------------------------------------------- memory
+constexpr int kMaxDevices = 64;              // per-device state (memory pools, function attributes)
 void* dalloc(size_t bytes, cudaStream_t s);  // nullptr on failure
 void dfree(void* p, cudaStream_t s);
 
@@ -117,6 +118,8 @@ cudaError_t cluster_fit(const double* raw, long long n, const int* init_idx, int
 cudaError_t cluster_vote(const ClusterModel* M, const int* labels, int* out, cudaStream_t s);
 cudaError_t cluster_predict(const ClusterModel* M, const double* raw, long long q, int* cluster, cudaStream_t s);
 ClusterModel* cluster_new();
+// eigen.cpp: leading k eigenpairs of a symmetric n x n matrix, descending, sign-normalised (F3)
+bool sym_eigen_basis(int n, const double* C, int k, double* basis, double* eigval);
 void cluster_free(ClusterModel* M);
 void cluster_info(const ClusterModel* M, sfs_cluster_info* out);
 

@@ -52,13 +52,13 @@ __device__ __forceinline__ void pdl_early() { pdl_trigger(); }
 __device__ __forceinline__ void pdl_early() {}
 #endif
 
+// Environment A/B switches are read once per process (thread-safe function-local statics).
 bool pdl_enabled() {
-  static int v = -1;
-  if (v < 0) {
+  static const bool v = [] {
     const char* e = getenv("SFS_PDL");
-    v = (e && e[0] == '0') ? 0 : 1;
-  }
-  return v == 1;
+    return !(e && e[0] == '0');
+  }();
+  return v;
 }
 
 // cudaLaunchKernelEx with the programmatic-stream-serialization attribute (PDL).
@@ -1347,14 +1347,15 @@ cudaError_t launch_csr_stream(const int* rp, const int* col, const T* val, const
 // consecutive-row DIA (k_spmv_dia_v4): fp32 by default (SFS_DIA_F4=0 disables), fp64 on request
 // (SFS_DIA_V4_F64=1) -- A/B switches
 bool dia_v4_enabled(size_t elem) {
-  static int f32 = -1, f64 = -1;
-  if (f32 < 0) {
+  static const bool f32 = [] {
     const char* e = getenv("SFS_DIA_F4");
-    f32 = (e && e[0] == '0') ? 0 : 1;
+    return !(e && e[0] == '0');
+  }();
+  static const bool f64 = [] {
     const char* d = getenv("SFS_DIA_V4_F64");
-    f64 = (d && d[0] == '1') ? 1 : 0;
-  }
-  return elem == 4 ? f32 == 1 : f64 == 1;
+    return d && d[0] == '1';
+  }();
+  return elem == 4 ? f32 : f64;
 }
 
 template <typename T, bool PUSH>
@@ -1367,11 +1368,10 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   // 0.73 -> 0.80); fp32 keeps the latency rule (its S = 1 is fastest)
   if (sizeof(T) == 8)
     while (S < 16 && A->ndiag / (2 * S) >= 12) S <<= 1;
-  static int force_s = -2;  // SFS_DIA_S: A/B override of the diagonal split (1, 2, 4, 8, 16)
-  if (force_s == -2) {
+  static const int force_s = [] {  // SFS_DIA_S: A/B override of the diagonal split (1, 2, 4, 8, 16)
     const char* e = getenv("SFS_DIA_S");
-    force_s = e ? atoi(e) : -1;
-  }
+    return e ? atoi(e) : -1;
+  }();
   if (force_s == 1 || force_s == 2 || force_s == 4 || force_s == 8 || force_s == 16) S = force_s;
   const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
   const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
@@ -1382,11 +1382,10 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   if (dia_v4_enabled(sizeof(T))) {
     // L2 prefetch of the next batch's slab (SFS_DIA_PF: distance in batches, 0 = off; A/B switch).
     // 128^3 fp32 stencil cold (tools/ab_dia_pf.sh): off 54.3 us (0.69), 1: 52.2 us (0.71), 2: 53.2, 3: 55.3
-    static int pfd = -1;
-    if (pfd < 0) {
+    static const int pfd = [] {
       const char* e = getenv("SFS_DIA_PF");
-      pfd = e ? atoi(e) : 1;
-    }
+      return e ? atoi(e) : 1;
+    }();
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
     switch (S) {
       case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
@@ -1430,11 +1429,10 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         // next-chunk L2 prefetch above SFS_TILE_PF_MB of footprint (default 256 = 2 x L2; < 0: never).
         // Cold, tools/ab_tile_pf.sh: 1M-row band fp64 0.81 -> 0.85 of peak; applied to every matrix the
         // corpus CSR race got 2.5 % slower (L2-resident matrices), hence the gate.
-        static long long pf_mb = -2;
-        if (pf_mb == -2) {
+        static const long long pf_mb = [] {
           const char* ev = getenv("SFS_TILE_PF_MB");
-          pf_mb = ev ? atoll(ev) : 256;
-        }
+          return ev ? atoll(ev) : 256LL;
+        }();
         const long long foot = 4 * (m + 1) + (4 + (long long)sizeof(T)) * z + (long long)sizeof(T) * (A->n + m);
         const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
         auto go = [&](auto kern) {
@@ -1569,13 +1567,14 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
 // the ELL-part -> COO-part pair.
 int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) {
   const long long o = nnz_max - K;
-  static long long small = -2, large = -2;  // SFS_HYB_ROWWISE="small,large": A/B overrides of the limits
-  if (small == -2) {
-    small = kHybRowwiseSmall;
-    large = kHybRowwiseLarge;
+  struct Lim { long long small, large; };
+  static const Lim lim = [] {  // SFS_HYB_ROWWISE="small,large": A/B overrides of the limits
+    Lim l{kHybRowwiseSmall, kHybRowwiseLarge};
     const char* e = getenv("SFS_HYB_ROWWISE");
-    if (e) sscanf(e, "%lld,%lld", &small, &large);
-  }
+    if (e) sscanf(e, "%lld,%lld", &l.small, &l.large);
+    return l;
+  }();
+  const long long small = lim.small, large = lim.large;
   return coo_nnz > 0 && (o <= large || (z < (1LL << 20) && o <= small));
 }
 

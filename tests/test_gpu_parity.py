@@ -10,7 +10,7 @@ import oracle
 import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
 import sfsgen
 from gpu_util import assert_features_equal, check_conversion, check_spmv, to_dev
-from helpers import golden, random_csr
+from helpers import golden, q11_boundary_cases, random_csr
 
 pytestmark = pytest.mark.gpu
 
@@ -376,3 +376,23 @@ def test_csr_bitmap_tile(dtype, cap):
     assert M.layout().variant == 3
     check_spmv(B, sfs.CSR, M, x[:B.n] if len(x) >= B.n else sfsgen.vector(6, B.n, B.dtype), B.dtype, ctx="bitmap-fallback")
     M.free()
+
+
+@pytest.mark.parametrize("name", ["slack_at", "slack_past", "fill_at_dia", "fill_past_dia", "fill_at_ell",
+                                  "fill_past_ell", "trunc_at", "trunc_past"])
+def test_q11_admissibility_boundary_gpu(name):
+    """The library's Q11 decision at E = lim and lim + 1 (Q11) equals the hand-derived bits (and
+    the oracle's features, bitwise); an inadmissible ELL / DIA conversion returns SFS_ERR_INADMISSIBLE."""
+    A, kw, e = q11_boundary_cases()[name]
+    opts = sfs.default_opts(**kw)
+    fg = sfs.features(to_dev(A), opts)
+    assert_features_equal(fg, oracle.features(A.m, A.n, A.rp, A.col, oracle.default_opts(**kw) if kw else None), name)
+    assert bool((fg["admissible_mask"] >> sfs.ELL) & 1) == e["ell_ok"]
+    assert bool((fg["admissible_mask"] >> sfs.DIA) & 1) == e["dia_ok"]
+    for fmt, ok in ((sfs.ELL, e["ell_ok"]), (sfs.DIA, e["dia_ok"])):
+        if ok:
+            sfs.convert(to_dev(A), fmt, opts).free()
+        else:
+            with pytest.raises(sfs.SfsError) as ei:
+                sfs.convert(to_dev(A), fmt, opts)
+            assert ei.value.status == sfs.ERR_INADMISSIBLE

@@ -1,5 +1,8 @@
-"""GPU parity of the semi-supervised predictor against the oracle chain:
-bit-exact ranges, PCA basis, centroids, assignments, votes and predictions."""
+"""GPU parity of the semi-supervised predictor against the oracle chain: ranges and
+means bit-exact (same fixed-order definitions); the PCA step is solved independently on each side
+(library: Householder + implicit QL, csrc/eigen.cpp, itself pinned to numpy eigh in tests/test_pca_pin.py;
+oracle: cyclic Jacobi), so eigenvalues / basis / centroids agree to a tolerance and the discrete results
+(assignments, iterations, votes, predictions) exactly."""
 import numpy as np
 import pytest
 
@@ -26,14 +29,22 @@ def _table(count, seed):
 
 
 @pytest.mark.parametrize("nc,pcs", [(6, 8), (20, 8), (9, 4)])
-def test_fit_vote_predict_bit_exact(nc, pcs):
+def test_fit_vote_predict_parity(nc, pcs):
     raw, labels, _ = _table(120, 5)
     init = np.random.default_rng(nc).choice(len(raw), size=nc, replace=False).astype(np.int32)
     ref = oracle.ss_fit(raw, init, pcs=pcs)
     M = sfs.ClusterModel(raw, init, pcs=pcs)
     g = M.info
-    for k in ("mins", "maxs", "mean", "basis", "eigval", "centroids"):
+    for k in ("mins", "maxs", "mean"):
         assert np.array_equal(g[k], ref[k]), k
+    scale = float(ref["eigval"][0])
+    assert np.abs(g["eigval"] - ref["eigval"]).max() <= 1e-12 * scale
+    ev_all = ref["eigval"]
+    for c in range(pcs):
+        gap = min(abs(ev_all[c] - ev_all[j]) for j in range(pcs) if j != c)
+        if gap > 1e-6 * scale:
+            assert np.abs(g["basis"][c] - ref["basis"][c]).max() <= 1e-9 * scale / gap, c
+    assert np.allclose(g["centroids"], ref["centroids"], rtol=0, atol=1e-10)
     assert (g["assign"] == ref["assign"]).all() and g["iters"] == ref["iters"]
     bench = labels.copy()
     bench[::3] = -1  # a third of the corpus not benchmarked

@@ -14,7 +14,7 @@ import pytest
 
 import oracle
 import sfsgen
-from helpers import (csr_max_closed_form, dense_of, exact_matvec, features_from_histogram, golden, kth_largest,
+from helpers import (q11_boundary_cases, csr_max_closed_form, dense_of, exact_matvec, features_from_histogram, golden, kth_largest,
                      pattern_of, random_csr, stencil_histogram, ulp_close)
 
 F = Fraction
@@ -192,6 +192,21 @@ def test_empty_and_degenerate():
     f = oracle.features(m, m, rp, col)
     assert f["ell_size"] == m * m and not (f["admissible_mask"] >> oracle.ELL) & 1
     assert (f["admissible_mask"] >> oracle.HYB) & 1
+
+
+@pytest.mark.parametrize("name", ["slack_at", "slack_past", "fill_at_dia", "fill_past_dia", "fill_at_ell",
+                                  "fill_past_ell", "trunc_at", "trunc_past"])
+def test_q11_admissibility_boundary(name):
+    """Q11 (CUSP size restrictions P:L194): ELL / DIA admissible iff padded slots E <=
+    max(trunc(max_fill * z), fill_slack).  Each case sits at E = lim or lim + 1, once where fill_slack
+    binds, once where trunc(3z) binds (for ELL and for DIA), once where trunc of a non-integer limit
+    decides; the expected bits are literal numbers derived by hand (tests/helpers.q11_boundary_cases)."""
+    A, kw, e = q11_boundary_cases()[name]
+    f = oracle.features(A.m, A.n, A.rp, A.col, oracle.default_opts(**kw) if kw else None)
+    assert (f["nnz"], f["ell_size"], f["dia_size"]) == (e["z"], e["ell_size"], e["dia_size"])
+    assert bool((f["admissible_mask"] >> oracle.ELL) & 1) == e["ell_ok"]
+    assert bool((f["admissible_mask"] >> oracle.DIA) & 1) == e["dia_ok"]
+    assert f["admissible_mask"] & 0b1011 == 0b1011  # CSR, COO, HYB always
 
 
 # ------------------------------------------------------------------ conversions: invariants

@@ -106,3 +106,71 @@ def test_kmeans_against_sklearn():
     # assignment = nearest centroid, ties to the lowest id
     tie = oracle.ss_assign(np.zeros((1, 8)), np.stack([np.ones(8), -np.ones(8)]))
     assert tie[0] == 0
+
+
+FRACTIONS = {"nnz_frac", "hyb_ell_frac", "dia_frac", "ell_frac"}  # F1: sqrt; every other Table-1 feature log1p
+
+
+def _np_transform(raw):
+    """F1 written independently from the reading: sqrt for the four fractions, log1p otherwise."""
+    out = np.empty_like(raw)
+    for j, name in enumerate(oracle.TABLE1):
+        out[:, j] = np.sqrt(raw[:, j]) if name in FRACTIONS else np.log1p(raw[:, j])
+    return out
+
+
+def _np_corpus(rng, n):
+    """Table-1-shaped rows: counts / sizes spanning decades, fractions in (0, 1]."""
+    raw = np.exp(rng.uniform(0, 14, size=(n, oracle.NFEAT)))
+    for j, name in enumerate(oracle.TABLE1):
+        if name in FRACTIONS:
+            raw[:, j] = rng.uniform(1e-6, 1.0, size=n)
+    return raw
+
+
+def test_scale_against_numpy():
+    """or_ss_scale (the prediction path's scaling, F2): queries transformed, then mapped with
+    the TRAINING ranges, unclipped (queries may leave [0, 1]); a constant training column maps to 0."""
+    rng = np.random.default_rng(11)
+    train = _np_corpus(rng, 120)
+    train[:, 4] = 3.0  # constant column
+    q = _np_corpus(rng, 40)
+    q[:3] *= 50.0  # beyond the training range
+    X, mins, maxs = oracle.ss_preprocess(train)
+    t = _np_transform(train)
+    # numpy's log1p may differ from the C library's by an ulp: compare to 1e-15 relative
+    assert np.allclose(mins, t.min(0), rtol=1e-15, atol=0) and np.allclose(maxs, t.max(0), rtol=1e-15, atol=0)
+    got = oracle.ss_scale(q, mins, maxs)
+    tq = _np_transform(q)
+    rng_ = t.max(0) - t.min(0)
+    want = np.where(rng_ > 0, (tq - t.min(0)) / np.where(rng_ > 0, rng_, 1.0), 0.0)
+    assert np.allclose(got, want, rtol=1e-13, atol=1e-13)
+    assert (got[:, 4] == 0).all()
+    assert got.max() > 1.0  # unclipped
+    # the training rows themselves map onto ss_preprocess's output
+    assert np.allclose(oracle.ss_scale(train, mins, maxs), X, rtol=0, atol=1e-15)
+
+
+def test_predict_against_numpy():
+    """ss_predict (a new matrix gets its nearest centroid's cluster): numpy recomputes scale ->
+    centre -> project on the fitted basis -> argmin squared distance (first index on ties) from the fit's
+    parameters; the oracle's cluster ids match wherever the two nearest centroids are not within
+    rounding of each other."""
+    rng = np.random.default_rng(12)
+    train = _np_corpus(rng, 300)
+    q = _np_corpus(rng, 200)
+    init = rng.choice(300, size=12, replace=False).astype(np.int32)
+    fit = oracle.ss_fit(train, init, pcs=8)
+    X = oracle.ss_scale(q, fit["mins"], fit["maxs"])
+    Y = (X - fit["mean"]) @ fit["basis"].T
+    d2 = ((Y[:, None, :] - fit["centroids"][None, :, :]) ** 2).sum(-1)
+    want = np.argmin(d2, axis=1)
+    srt = np.sort(d2, axis=1)
+    clear = srt[:, 1] - srt[:, 0] > 1e-9 * (1 + srt[:, 0])
+    got = oracle.ss_predict(fit, q)
+    assert clear.sum() > 190
+    assert (got[clear] == want[clear]).all()
+    # the fitted training assignment is the same rule applied to the training rows
+    Yt = (oracle.ss_scale(train, fit["mins"], fit["maxs"]) - fit["mean"]) @ fit["basis"].T
+    d2t = ((Yt[:, None, :] - fit["centroids"][None, :, :]) ** 2).sum(-1)
+    assert (np.argmin(d2t, axis=1) == fit["assign"]).mean() > 0.99
