@@ -1,12 +1,17 @@
 #!/usr/bin/env python
 """bench.py — matrices labelled per second on the BASELINE configs[1] corpus (the headline metric).
 
-One step = the whole hot path (SURVEY §8(a) a1–a15) over one batch: for every matrix of the rank's
-corpus-200 (configs[1]: banded / uniform random / block-diagonal / power-law, 10K–1M rows, fp32 and
+One step = the whole hot path (SURVEY §8(a) a1–a15) over one batch: for every matrix of the
+configs[1] corpus-200 (banded / uniform random / block-diagonal / power-law, 10K–1M rows, fp32 and
 fp64 values) the Table-1 feature pass, every admissible conversion, the device-timed format race
-(5 warm-up + 100 timed SpMVs per format) and the label; at N > 1 the labels/features are
-gathered over NCCL.  Inputs are resident in HBM when the timed region starts (`value`); `e2e`
-repeats the step through the same C-ABI call with pinned HOST buffers (H2D inside the call).
+(5 warm-up + 100 timed SpMVs per format) and the label, then the all-gather of every rank's
+fixed-size result rows (inside the timed region).  At N GPUs the SAME 200 matrices are LPT-sharded
+over the ranks on an estimated race cost (strong scaling: "Scaling = rate(P)/rate(1) on
+the identical corpus and seeds"; --scaling weak gives every rank its own 200).  Inputs are resident in
+HBM when the timed region starts (`value`); `e2e` repeats the step through the same C-ABI call with
+pinned HOST buffers (H2D inside the call).  The `rowpart` record times BASELINE configs[3] (3D
+27-point stencil, 128^3, fp64) row-partitioned over the N ranks with each exchange of SURVEY §8(e) 2 /
+§8(f) f3 (NCCL all-gather of x, NCCL halo send/recv, push fused into the SpMV over peer memory).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
@@ -52,6 +57,10 @@ def parse():
     p.add_argument("--dump", default=None, help="write per-matrix results of the last timed step (JSONL)")
     p.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                    help="gloo: host-side collectives, lets N ranks share one GPU (tests of the N > 1 path only)")
+    p.add_argument("--scaling", default="strong", choices=["strong", "weak"],
+                   help="strong: the identical corpus-200 sharded over the N ranks; weak: 200 matrices per rank")
+    p.add_argument("--rowpart-N", type=int, default=128, help="configs[3] grid edge (0 = skip the rowpart record)")
+    p.add_argument("--rowpart-iters", type=int, default=100)
     return p.parse_args()
 
 
@@ -62,11 +71,18 @@ def dist_env():
     return rank, world, local
 
 
-def corpus_ids(rank, per_rank, world=1):
-    """Weak scaling: the job is the first per_rank*world matrices of the configs[1] recipe, LPT-balanced
-    over the ranks on an estimated race cost (dist.weak_shard); N = 1 labels ids [0, per_rank)."""
+def corpus_ids(rank, per_rank, world=1, scaling="strong"):
+    """strong: the first per_rank matrices of the configs[1] recipe (200: the whole corpus), LPT-sharded over
+    the ranks on an estimated race cost (dist.race_cost; identical on every rank, no communication).
+    weak: the first per_rank*world matrices, LPT-balanced so every rank gets ~per_rank (dist.weak_shard)."""
+    import sfsgen
     from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
-    return sd.weak_shard(200, per_rank, rank, world)
+    if scaling == "weak":
+        return sd.weak_shard(200, per_rank, rank, world)
+    ids = list(range(per_rank))
+    if world == 1:
+        return ids
+    return [ids[j] for j in sd.lpt_assign([sd.race_cost(sfsgen.corpus_spec(200, i)) for i in ids], world)[rank]]
 
 
 def generate_host(ids):
@@ -132,29 +148,39 @@ class ClockSampler:
 
 
 # ------------------------------------------------------------------ CPU oracle (cpu_baseline / reference arm)
+def stratified(items, stride=9):
+    """Corpus order interleaved with a stride (ids 0, 9, 18, ..., 1, 10, ...; 9 is coprime with the 4 classes
+    of i mod 4): a bounded prefix spans the size range, the four classes and both value types of corpus-200
+    instead of its first few matrices."""
+    return [items[j] for r in range(stride) for j in range(r, len(items), stride)]
+
+
 def oracle_sample(host_mats, budget_s, threads, reps_target=100, reps_cpu=3):
-    """The oracle's whole labelling pass (features, every admissible conversion, timed SpMV reps per
-    format, argmin) on the matrices in corpus order, `threads` matrices at a time, dispatching until
-    `budget_s` of wall time is spent.  Each matrix runs `reps_cpu` SpMV reps per format; its
-    single-thread time is scaled to `reps_target` reps with its own measured per-rep SpMV times:
-        t_i = wall_i + (reps_target - reps_cpu) * sum_f t_spmv_f,i
-    and the throughput is threads * done / sum_i t_i (perfect scaling over cores: generous to the CPU).
-    Returns (matrices/s, done, threads, wall, nnz, measured matrices/s at reps_cpu)."""
+    """The oracle's whole labelling pass (features, every admissible conversion, `reps_cpu` timed SpMV reps
+    per format, argmin) on the matrices in stratified order, `threads` matrices at a time (one thread
+    each), dispatching until `budget_s` of wall time is spent.  Each matrix's time is its own measured
+    wall time under that load, with the SpMV reps scaled to `reps_target` by its own measured per-rep
+    times:  t_i = wall_i + (reps_target - reps_cpu) * sum_f t_spmv_f,i.
+    Throughput = threads * done / sum_i t_i: the per-matrix times are MEASURED with `threads` jobs
+    running concurrently (memory-bandwidth contention included); only a perfectly load-balanced long
+    corpus is assumed.  Returns (matrices/s, done, threads, wall, nnz, per-matrix times in sample order)."""
     import oracle
     from concurrent.futures import ThreadPoolExecutor, FIRST_COMPLETED, wait
 
     t0 = time.perf_counter()
     done, nnz, tsum = 0, 0, 0.0
-    it = iter(host_mats)
+    order = stratified(host_mats)
+    it = iter(enumerate(order))
+    times = {}
     futs = set()
 
     def job(item):
-        _, A, x = item
+        k, (_, A, x) = item
         w0 = time.perf_counter()
         _, _, ts, _ = oracle.label_matrix(A.m, A.n, A.rp, A.col, A.val.astype(np.float64), x.astype(np.float64),
                                           reps=reps_cpu)
         wall_i = time.perf_counter() - w0
-        return A.nnz, wall_i + (reps_target - reps_cpu) * float(np.sum(ts))
+        return k, A.nnz, wall_i + (reps_target - reps_cpu) * float(np.sum(ts))
 
     with ThreadPoolExecutor(max_workers=threads) as ex:
         for _ in range(threads):
@@ -165,7 +191,8 @@ def oracle_sample(host_mats, budget_s, threads, reps_target=100, reps_cpu=3):
         while futs:
             fin, futs = wait(futs, return_when=FIRST_COMPLETED)
             for f in fin:
-                z, ti = f.result()
+                k, z, ti = f.result()
+                times[k] = ti
                 nnz += z
                 tsum += ti
                 done += 1
@@ -175,7 +202,31 @@ def oracle_sample(host_mats, budget_s, threads, reps_target=100, reps_cpu=3):
                     if nxt is not None:
                         futs.add(ex.submit(job, nxt))
     wall = time.perf_counter() - t0
-    return threads * done / tsum, done, threads, wall, nnz, done / wall
+    return threads * done / tsum, done, threads, wall, nnz, [times[k] for k in sorted(times)]
+
+
+def cpu_baseline_record(host_mats, budget_s, reps):
+    """T = nproc (the reported value) and T = 1 (BASELINE.md CPU plan).  T = nproc as oracle_sample says.
+    T = 1: the first matrices of the same stratified order, one job alone on the machine; its rate is put on
+    the T = nproc sample by the measured ratio of single-job to under-load per-matrix times on the matrices
+    both runs labelled (so both figures describe the same sample)."""
+    nproc = os.cpu_count() or 1
+    v, d, c, w, nnz, tn = oracle_sample(host_mats, budget_s, nproc, reps_target=reps)
+    _, d1, _, w1, nnz1, t1 = oracle_sample(host_mats, max(3.0, budget_s / 3), 1, reps_target=reps)
+    common = min(d1, len(tn))
+    r = sum(t1[:common]) / sum(tn[:common]) if common else float("nan")  # single-job / under-load time
+    v1 = (len(tn) / (r * sum(tn))) if common else None
+    sample = (f"stratified sample (every 9th matrix first) of corpus-200: T={c}: {d} matrices ({nnz} nnz), "
+              f"{w:.1f} s wall; T=1: the first {d1} of them ({nnz1} nnz) alone, {w1:.1f} s wall.  Oracle labelling "
+              f"pass per matrix (features + every admissible conversion + 3 SpMV reps per format + argmin), each "
+              f"matrix's SpMV reps scaled to {reps} by its own measured per-rep times; T={c}: per-matrix times "
+              f"measured with {c} jobs running concurrently (one thread each), throughput = {c} x matrices / sum of "
+              f"times (perfect load balance over a long corpus assumed, contention measured)")
+    return {"value": v, "unit": UNIT, "cores": c, "kind": "oracle", "sample": sample,
+            "t1": {"value": v1, "unit": UNIT, "cores": 1, "matrices_measured": d1,
+                   "single_job_over_loaded_time": r,
+                   "note": "T=1 rate on the T=nproc sample: matrices / (sum of under-load times x measured ratio)"},
+            "speedup_t1_to_tn": v / v1 if v1 else None}
 
 
 def run_reference(args):
@@ -194,17 +245,184 @@ def run_reference(args):
         walls.append(w)
         done.append(d)
     value = statistics.median(vals)
-    sample = (f"first {min(done)}-{max(done)} matrices (corpus order) of corpus-200 per step, oracle labelling "
-              f"pass (features + conversions + 3 SpMV reps/format + argmin) with each matrix's time scaled to "
-              f"{args.reps} reps by its own per-rep SpMV time; {threads} threads, perfect core scaling assumed")
+    sample = (f"{min(done)}-{max(done)} matrices of corpus-200 per step in stratified order (every 9th first), "
+              f"oracle labelling pass (features + conversions + 3 SpMV reps/format + argmin), each matrix's SpMV "
+              f"reps scaled to {args.reps} by its own measured per-rep times; {threads} concurrent single-thread "
+              f"jobs, throughput = {threads} x matrices / sum of the measured per-matrix times")
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1000 * statistics.median(walls),
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": {"workload": "corpus-200 (BASELINE configs[1])", "matrices_per_rank": args.corpus},
+            "higher_is_better": True, "scaling": "strong" if args.scaling == "strong" else "weak",
+            "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": "corpus-200 (BASELINE configs[1])", "matrices": args.corpus},
             "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
+
+
+# ------------------------------------------------------------------ configs[3] row partition (rowpart record)
+def rowpart_measure(N, iters, warmup, rank, world, dev, gloo, group=None, formats=("DIA", "CSR")):
+    """BASELINE configs[3]: the 3D 27-point stencil on an N^3 grid (fp64), rows partitioned into `world`
+    equal contiguous blocks.  Per format, per exchange, `warmup` untimed then `iters`
+    timed power-iteration steps (y becomes the next x) between CUDA events on the launching stream, max
+    over ranks (SURVEY §8(d) "Row partition (C4)"):
+      allgather: all_gather_into_tensor(x_full, x_local) + sfs_spmv of the block (global column ids);
+      halo:      NCCL send/recv of the ghost entries only (sfs_gather packs) + sfs_spmv of the renumbered
+                 block (SURVEY §8(f) f3);
+      push:      sfs_spmv_push -- the ghost rows stored into the neighbours' next x by the SpMV kernel
+                 itself over CUDA-IPC peer memory (NVLink), flags instead of NCCL (§8(f) f3).
+    Also the all-gather alone, the block SpMV alone, and (rank 0) the whole matrix's SpMV on one GPU, so
+    efficiency = t_spmv_full(1 GPU) / (P * t_iter(P)) is computed inside the run.  gloo (ranks sharing
+    one GPU, tests only): the all-gather goes through host memory; halo is skipped."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    import sfsgen
+    from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
+
+    A = sfsgen.stencil3d27(N, dtype=sfsgen.F64)  # host, untimed (every rank: the slice needs row_ptr)
+    part = sd.RowPartition(A.m, A.n, world, rank)
+    b = part.bounds
+    rp, col, val = sd.slice_rows(A.rp, A.col, A.val, b[rank], b[rank + 1])
+    t = lambda a: torch.from_numpy(np.ascontiguousarray(a)).to(dev)
+    x0 = sfsgen.vector(5, A.n)
+    x_local = t(x0[b[rank]:b[rank + 1]])
+    stream = torch.cuda.current_stream()
+    cdev = torch.device("cpu") if gloo else dev
+
+    def barrier():
+        if world > 1:
+            dist.barrier(group=group)
+        torch.cuda.synchronize()
+
+    def maxr(v):
+        if world == 1:
+            return v
+        tt = torch.tensor([v], dtype=torch.float64, device=cdev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX, group=group)
+        return float(tt.item())
+
+    def sumr(v):
+        if world == 1:
+            return v
+        tt = torch.tensor([v], dtype=torch.float64, device=cdev)
+        dist.all_reduce(tt, op=dist.ReduceOp.SUM, group=group)
+        return float(tt.item())
+
+    def timed(fn, n):
+        """seconds per iteration of fn(n), CUDA events on the launching stream, max over ranks"""
+        fn(warmup)
+        barrier()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        fn(n)
+        e1.record(stream)
+        barrier()
+        return maxr(e0.elapsed_time(e1) / 1000.0 / n)
+
+    blk = part.block
+    x_pad = torch.zeros(blk, dtype=torch.float64, device=dev)
+    x_full = torch.empty(blk * world, dtype=torch.float64, device=dev)
+
+    def allgather(dst, src):
+        if world == 1:
+            dst.copy_(src)
+        elif gloo:  # tests only: host staging
+            h = torch.empty(dst.numel(), dtype=dst.dtype)
+            dist.all_gather_into_tensor(h, src.cpu(), group=group)
+            dst.copy_(h)
+        else:
+            dist.all_gather_into_tensor(dst, src, group=group)
+
+    halo_ok = world == 1 or not gloo
+    plan = sd.halo_plan(part, col, group=group, device=cdev)  # world 1: no ghosts
+    out = {"config": f"BASELINE configs[3]: 3D 27-point stencil {N}^3 (m = {A.m}, nnz = {A.nnz}), fp64, "
+                     f"{world} contiguous row blocks of {blk} rows", "n_gpus": world, "iters": iters,
+           "warmup": warmup, "halo_entries_per_rank_max": int(maxr(float(plan.recv_count))),
+           "allgather_entries_per_rank": int(blk * (world - 1)), "formats": {}}
+    y_loc = torch.empty(part.local_rows, dtype=torch.float64, device=dev)
+    for fname in formats:
+        fmt = sfs.FORMAT_NAMES.index(fname)
+        rec = {}
+        # global-column block (all-gather path)
+        Ak = sfs.Csr(part.local_rows, A.n, t(rp), t(col), t(val))
+        M = sfs.convert(Ak, fmt)
+        fk = sfs.features(Ak)
+        nbytes = sfs.spmv_bytes(fk, fmt, sfs.F64)
+        rec["kernel_variant"] = M.layout().variant
+
+        def ag_iter(n):
+            cur = x_local
+            for _ in range(n):
+                x_pad[:cur.numel()].copy_(cur)
+                allgather(x_full, x_pad)
+                sfs.spmv(fmt, M, x_full[:A.n], y_loc)
+                cur = y_loc
+
+        def ag_only(n):
+            for _ in range(n):
+                allgather(x_full, x_pad)
+
+        def mv_only(n):
+            for _ in range(n):
+                sfs.spmv(fmt, M, x_full[:A.n], y_loc)
+
+        x_pad[:x_local.numel()].copy_(x_local)
+        allgather(x_full, x_pad)
+        rec["allgather"] = {"t_iter_us": 1e6 * timed(ag_iter, iters)}
+        rec["t_allgather_only_us"] = 1e6 * timed(ag_only, iters)
+        rec["t_spmv_only_us"] = 1e6 * timed(mv_only, iters)
+        M.free()
+        # renumbered block (halo and push paths)
+        Mh = sfs.convert(sfs.Csr(part.local_rows, plan.n_ext, t(rp), t(plan.col_ext), t(val)), fmt)
+        if halo_ok:
+            spmv_h = lambda xe, yv: sfs.spmv(fmt, Mh, xe, yv)
+            rec["halo"] = {"t_iter_us": 1e6 * timed(
+                lambda n: sd.rowpart_halo_iterate(plan, spmv_h, sfs.gather, x_local, n, group=group), iters)}
+        else:
+            rec["halo"] = {"skipped": "gloo test mode (NCCL send/recv of device buffers)"}
+        try:
+            tm = {}
+            sd.rowpart_push_iterate(plan, Mh, fmt, x_local, warmup, group=group)
+            barrier()
+            sd.rowpart_push_iterate(plan, Mh, fmt, x_local, iters, group=group, timing=tm)
+            rec["push"] = {"t_iter_us": 1e3 * maxr(tm["ms_per_iter"]), "transport": "CUDA IPC peer memory"}
+        except Exception as ex:  # report, never hide
+            rec["push"] = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+        Mh.free()
+        tot_bytes = sumr(float(nbytes))
+        rec["spmv_bytes_all_ranks"] = tot_bytes
+        # whole matrix on one GPU (rank 0): the P = 1 reference of the efficiency
+        t1 = 0.0
+        if rank == 0:
+            Af = sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val))
+            Mf = sfs.convert(Af, fmt)
+            xf = t(x0)
+            yf = torch.empty(A.m, dtype=torch.float64, device=dev)
+
+            def full(n):
+                for _ in range(n):
+                    sfs.spmv(fmt, Mf, xf, yf)
+            full(warmup)
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            full(iters)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            t1 = e0.elapsed_time(e1) / 1000.0 / iters
+            Mf.free()
+            del Af, xf, yf
+        t1 = maxr(t1)
+        rec["t_spmv_full_matrix_1gpu_us"] = 1e6 * t1
+        for ex in ("allgather", "halo", "push"):
+            ti = rec[ex].get("t_iter_us")
+            if ti:
+                rec[ex]["agg_gbs"] = tot_bytes / (ti / 1e6) / 1e9
+                rec[ex]["efficiency"] = (1e6 * t1) / (world * ti)
+        out["formats"][fname] = rec
+    return out
 
 
 # ------------------------------------------------------------------ our arm
@@ -213,6 +431,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    from paper_conf_icppw_dhandhaniadpbl21_b200 import dist as sd
 
     rank, world, local = dist_env()
     local = local % torch.cuda.device_count()
@@ -227,7 +446,7 @@ def run_ours(args):
     cdev = torch.device("cpu") if gloo else dev  # where the collectives' tensors live
     stream = torch.cuda.current_stream()
 
-    host = generate_host(corpus_ids(rank, args.corpus, world))
+    host = generate_host(corpus_ids(rank, args.corpus, world, args.scaling))
     t = lambda a: torch.from_numpy(a).to(dev)
     mats = [sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), t(x)) for _, A, x in host]
     pin = lambda a: torch.from_numpy(a).pin_memory()
@@ -236,20 +455,28 @@ def run_ours(args):
     opts = sfs.default_opts(reps=args.reps, warmup=args.race_warmup, use_graphs=1 if args.graphs else 0)
     n = len(mats)
     n_max = n
-    if world > 1:  # LPT shards differ by a matrix or two: pad the gathered result rows
+    if world > 1:  # LPT shards differ in length: pad the gathered result rows
         nt = torch.tensor([n], dtype=torch.int64, device=cdev)
         dist.all_reduce(nt, op=dist.ReduceOp.MAX)
         n_max = int(nt.item())
-    gather_buf = torch.full((n_max * 9,), -1.0, dtype=torch.float64, device=cdev)
-    all_buf = torch.zeros(world * n_max * 9, dtype=torch.float64, device=cdev)
+    RF = sd.RESULT_FIELDS
+    gather_host = torch.full((max(n_max, 1), RF), -1.0, dtype=torch.float64).pin_memory()
+    gather_buf = torch.empty(max(n_max, 1) * RF, dtype=torch.float64, device=cdev)
+    all_buf = torch.zeros(world * max(n_max, 1) * RF, dtype=torch.float64, device=cdev)
+    gathered = {}
 
     def step(batch):
         feats, labs = sfs.label_corpus(batch, opts)
-        if world > 1:  # a15: gather labels + timing summary to every rank (results, ~64 B / matrix)
-            rows = [[i, L["label"]] + L["t_spmv_us"] + [L["t_features_us"], L["matrix_status"]]
-                    for (i, _, _), L in zip(host, labs)]
-            gather_buf[:n * 9].copy_(torch.tensor(rows, dtype=torch.float64).reshape(-1))
+        # a15: every rank's fixed-size result rows (id, label, statuses, times, 23 features) to every rank
+        rows = np.stack([sd.pack_result(i, f, L) for (i, _, _), f, L in zip(host, feats, labs)]) if n else None
+        if rows is not None:
+            gather_host[:n].copy_(torch.from_numpy(rows))
+        gather_buf.copy_(gather_host.reshape(-1), non_blocking=True)
+        if world > 1:
             dist.all_gather_into_tensor(all_buf, gather_buf)
+        else:
+            all_buf.copy_(gather_buf)
+        gathered["buf"] = all_buf
         return feats, labs
 
     def barrier():
@@ -297,9 +524,13 @@ def run_ours(args):
     total_mats = n_all * args.steps
     value = total_mats / t_max
     launches_all = int(sumr(float(launches)))
+    # the gathered rows hold every matrix of the job exactly once
+    got = gathered["buf"].reshape(-1, RF)[:, 0].cpu().numpy()
+    gathered_ids = sorted(int(v) for v in got if v >= 0)
+    gather_ok = len(gathered_ids) == n_all and len(set(gathered_ids)) == n_all
 
     # ---- e2e: same call with pinned host inputs (H2D inside the call), result D2H inside; one untimed
-    # warm-up step first (it grows the stream-ordered pool to hold the staged corpus)
+    # warm-up step first (it grows the pool to hold the staged corpus)
     if args.e2e_steps > 0:
         step(hmats)
     barrier()
@@ -315,7 +546,8 @@ def run_ours(args):
     e2e = None
     if args.e2e_steps > 0:
         e2e = {"value": n_all * args.e2e_steps / t_e2e, "unit": UNIT, "h2d_bytes_per_step": h2d,
-               "d2h_bytes_per_step": n * DAGGR_BYTES}
+               "d2h_bytes_per_step": n * DAGGR_BYTES,
+               "note": "per rank; H2D of the rank's CSR + x from pinned host memory inside sfs_label_corpus"}
 
     # ---- roofline of the dominant kernel (from the race's own CUDA events, inside the timed region)
     feats, labs = results[-1]
@@ -409,34 +641,41 @@ def run_ours(args):
                         "and L2-bound rather than HBM-bound; achieved_footprint_gt_2xL2 restricts to footprints "
                         "> 256 MB"}
 
+    # ---- configs[3] row partition over the same ranks (BASELINE configs[3])
+    rowpart = None
+    if args.rowpart_N > 0:
+        try:
+            rowpart = rowpart_measure(args.rowpart_N, args.rowpart_iters, 10, rank, world, dev, gloo)
+        except Exception as ex:  # reported in the line, never silently dropped
+            rowpart = {"error": f"{type(ex).__name__}: {ex}"[:400]}
+
     # ---- CPU oracle baseline (rank 0, N = 1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        threads = os.cpu_count() or 1
-        v, d, c, w, nnz, meas = oracle_sample(host, args.cpu_budget, threads, reps_target=args.reps)
-        cpu = {"value": v, "unit": UNIT, "cores": c, "kind": "oracle",
-               "sample": f"first {d} of this rank's {n} corpus-200 matrices in corpus order ({nnz} nnz): oracle "
-                         f"labelling pass (features + conversions + 3 SpMV reps/format + argmin), each matrix's time "
-                         f"scaled to {args.reps} reps by its own per-rep SpMV time; {c} threads, perfect core scaling "
-                         f"assumed; {w:.1f} s wall ({meas:.1f} matrices/s measured at 3 reps)"}
+        cpu = cpu_baseline_record(host, args.cpu_budget, args.reps)
 
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": 1000 * t_max / args.steps,
                 "step_ms": {"median": statistics.median(step_ms), "min": min(step_ms), "max": max(step_ms)},
                 "higher_is_better": True,
-                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+                "scaling": args.scaling, "vs_baseline": None, "dtype": "f64", "data": "synthetic",
                 "config": {"workload": "corpus-200 (BASELINE configs[1]): banded/uniform/block-diagonal/power-law, "
-                                       "10K-1M rows, values fp32 and fp64 (half each), SpMV accumulates in fp64",
-                           "matrices_per_rank": n, "matrices_all_ranks": n_all,
-                           "nnz_per_rank": int(sum(m.nnz for m in mats)),
+                                       "10K-1M rows, values fp32 and fp64 (half each); dtype = the SpMV arithmetic "
+                                       "(fp64 products and sums for both value types, y rounded once)",
+                           "matrices_rank0": n, "matrices_all_ranks": n_all,
+                           "nnz_rank0": int(sum(m.nnz for m in mats)),
                            "reps": args.reps, "race_warmup": args.race_warmup,
-                           "parallelism": f"corpus of {n_all} matrices LPT-sharded over {world} GPU(s) on estimated race "
-                                          f"cost (weak: {args.corpus} per GPU), no data-path collective",
+                           "parallelism": (f"the identical {n_all}-matrix corpus LPT-sharded over {world} GPU(s) on "
+                                           f"estimated race cost (strong scaling)" if args.scaling == "strong" else
+                                           f"{n_all} matrices, ~{args.corpus} per GPU (weak scaling)") +
+                                          "; one all_gather_into_tensor of 44-double result rows per step, timed",
+                           "gather_ok": gather_ok,
                            "l2": "inputs larger than L2 (corpus >> 126 MB per step); in-race reps back-to-back (P:L217)"},
                 "e2e": e2e, "gpu_launches": launches_all, "clocks": clk, "roofline": roofline,
                 "cpu_baseline": cpu, "per_format": per_fmt,
-                "label_histogram": {k: v["labels"] for k, v in per_fmt.items()}}
+                "label_histogram": {k: v["labels"] for k, v in per_fmt.items()},
+                "rowpart": rowpart}
         s = json.dumps(line)
         print(s, flush=True)
         if args.out:

@@ -173,7 +173,7 @@ def use_torch_allocator(enable: bool = True):
         L.sfs_set_allocator(cbs[0], cbs[1])
         _alloc_state["on"] = True
     elif not enable and _alloc_state["on"]:
-        L.sfs_set_allocator(None, None)
+        L.sfs_set_allocator(_ALLOC_T(), _FREE_T())  # NULL pointers: back to the library pool
         _alloc_state["on"] = False
 
 

@@ -80,9 +80,11 @@ def test_sharded_corpus_driver_single_rank():
         assert 0 <= r["label"] < 5 and r["matrix_status"] == 0
 
 
-def test_bench_two_ranks_share_one_gpu():
-    """bench.py's N > 1 path end to end (LPT weak shards, result all-gather, max-over-ranks timing,
-    summed launch counts): torchrun with 2 ranks on this one GPU, gloo collectives on host tensors."""
+@pytest.mark.parametrize("scaling", ["strong", "weak"])
+def test_bench_two_ranks_share_one_gpu(scaling):
+    """bench.py's N > 1 path end to end (LPT shards of the identical corpus or weak shards, the timed result
+    all-gather, max-over-ranks timing, summed launch counts, the configs[3]-shaped rowpart record at a small
+    grid with its all-gather and push exchanges): torchrun with 2 ranks on this one GPU, gloo collectives."""
     import json
     import os
     import socket
@@ -96,15 +98,23 @@ def test_bench_two_ranks_share_one_gpu():
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(root, "bench.py"),
            "--gpus", "2", "--steps", "1", "--warmup", "1", "--corpus", "6", "--e2e-steps", "1",
-           "--no-cpu-baseline", "--dist-backend", "gloo"]
+           "--no-cpu-baseline", "--dist-backend", "gloo", "--scaling", scaling, "--rowpart-N", "24",
+           "--rowpart-iters", "5"]
     r = subprocess.run(cmd, cwd=root, capture_output=True, text=True, timeout=900)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout[-2000:]
     d = json.loads(lines[0])
-    assert d["n_gpus"] == 2 and d["config"]["matrices_all_ranks"] == 12
+    assert d["n_gpus"] == 2 and d["config"]["matrices_all_ranks"] == (6 if scaling == "strong" else 12)
     assert d["value"] > 0 and d["e2e"]["value"] > 0 and d["gpu_launches"] > 0
-    assert d["scaling"] == "weak"
+    assert d["scaling"] == scaling and d["config"]["gather_ok"]
+    rp = d["rowpart"]
+    assert "error" not in rp, rp
+    for f in ("DIA", "CSR"):
+        r = rp["formats"][f]
+        assert r["allgather"]["t_iter_us"] > 0 and r["t_spmv_only_us"] > 0 and r["t_spmv_full_matrix_1gpu_us"] > 0
+        assert r["push"].get("t_iter_us", 0) > 0, r["push"]
+        assert "skipped" in r["halo"]
 
 
 def test_gather_kernel():
