@@ -61,6 +61,7 @@ def parse():
                    help="strong: the identical corpus-200 sharded over the N ranks; weak: 200 matrices per rank")
     p.add_argument("--rowpart-N", type=int, default=128, help="configs[3] grid edge (0 = skip the rowpart record)")
     p.add_argument("--rowpart-iters", type=int, default=100)
+    p.add_argument("--predictor-nc", type=int, default=20, help="clusters of the f2 subset-labelling record (0 = skip)")
     return p.parse_args()
 
 
@@ -641,6 +642,25 @@ def run_ours(args):
                         "and L2-bound rather than HBM-bound; achieved_footprint_gt_2xL2 restricts to footprints "
                         "> 256 MB"}
 
+    # ---- f2 / f4: cluster-subset labelling of the same corpus (N = 1): features of all, K-Means on them,
+    # race only one representative per cluster, vote, predict; scored against this step's full race
+    predictor = None
+    if world == 1 and args.predictor_nc > 0:
+        from paper_conf_icppw_dhandhaniadpbl21_b200 import predictor as pr
+        try:
+            r = pr.subset_labelling(mats, opts, nc=args.predictor_nc, k=1, truth=labs)
+            t_full = t_dev / args.steps
+            predictor = {k: r[k] for k in ("n", "nc", "k", "raced", "t_features_s", "t_fit_s", "t_subset_race_s",
+                                           "others_not_raced", "quality")}
+            predictor["t_full_race_s"] = t_full
+            predictor["race_time_saved"] = 1.0 - r["t_subset_race_s"] / t_full
+            predictor["time_saved_incl_clustering"] = 1.0 - r["t_total_s"] / t_full
+            predictor["note"] = ("PAPER.md L134/L167-169: only one matrix per cluster benchmarked; times device-measured "
+                                 "(CUDA events); t_subset_race_s = features of all + race of the representatives; "
+                                 "quality (P:L231 GT / CSR / Threshold, accuracy) against this run's full race")
+        except Exception as ex:
+            predictor = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+
     # ---- configs[3] row partition over the same ranks (BASELINE configs[3])
     rowpart = None
     if args.rowpart_N > 0:
@@ -675,7 +695,7 @@ def run_ours(args):
                 "e2e": e2e, "gpu_launches": launches_all, "clocks": clk, "roofline": roofline,
                 "cpu_baseline": cpu, "per_format": per_fmt,
                 "label_histogram": {k: v["labels"] for k, v in per_fmt.items()},
-                "rowpart": rowpart}
+                "predictor": predictor, "rowpart": rowpart}
         s = json.dumps(line)
         print(s, flush=True)
         if args.out:

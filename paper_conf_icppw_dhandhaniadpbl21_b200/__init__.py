@@ -131,18 +131,33 @@ EXPORTED = ["sfs_features", "sfs_convert", "sfs_spmv", "sfs_label_corpus", "sfs_
 # ------------------------------------------------------------------ allocator hook (§8(b) ownership)
 # Library-owned buffers (converted matrices, race temporaries, staged inputs) come from torch's caching
 # allocator, so they share one pool with the caller's tensors.  The library frees stream-ordered on the
-# stream it names; torch's allocator reuses a block on the stream it was allocated on, so a free on a
-# different stream first makes the allocation stream wait for the freeing stream (no reuse while the
-# freeing stream's kernels may still read the block).  SFS_TORCH_ALLOC=0 keeps the library's own CUDA
-# stream-ordered pool.
+# stream it names.  torch's allocator reuses a block on the stream it was allocated on, so a block freed
+# on ANOTHER stream (host inputs are staged on the copy stream and released on the compute stream) is
+# handed back only once an event recorded on the freeing stream has completed (the deferred-free
+# discipline of torch's record_stream; nothing waits, so the copy / race overlap is kept).
+# SFS_TORCH_ALLOC=0 keeps the library's own CUDA stream-ordered pool.
 _ALLOC_T = ctypes.CFUNCTYPE(_P, ctypes.c_size_t, _P)
 _FREE_T = ctypes.CFUNCTYPE(None, _P, _P)
-_alloc_state = {"on": False, "blocks": {}, "cbs": None}
+_alloc_state = {"on": False, "blocks": {}, "pending": [], "cbs": None}
+
+
+def _drain_pending(force=False):
+    import torch
+    pend = _alloc_state["pending"]
+    keep = []
+    for ev, ptr in pend:
+        if force or ev.query():
+            torch.cuda.caching_allocator_delete(ptr)
+        else:
+            keep.append((ev, ptr))
+    _alloc_state["pending"] = keep
 
 
 def _torch_alloc(nbytes, stream):
     try:
         import torch
+        if _alloc_state["pending"]:
+            _drain_pending()
         dev = torch.cuda.current_device()
         p = torch.cuda.caching_allocator_alloc(int(nbytes), dev, stream or 0)
         _alloc_state["blocks"][p] = (stream or 0, dev)
@@ -156,10 +171,14 @@ def _torch_free(ptr, stream):
         import torch
         a_stream, dev = _alloc_state["blocks"].pop(ptr, (stream or 0, None))
         if (stream or 0) != a_stream:
-            sa = torch.cuda.ExternalStream(a_stream, device=dev) if a_stream else torch.cuda.default_stream(dev)
             sf = torch.cuda.ExternalStream(stream, device=dev) if stream else torch.cuda.default_stream(dev)
-            sa.wait_stream(sf)
-        torch.cuda.caching_allocator_delete(ptr)
+            ev = torch.cuda.Event()
+            ev.record(sf)
+            _alloc_state["pending"].append((ev, ptr))
+        else:
+            torch.cuda.caching_allocator_delete(ptr)
+        if _alloc_state["pending"]:
+            _drain_pending()
     except Exception:
         pass
 

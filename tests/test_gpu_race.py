@@ -134,3 +134,26 @@ def test_mixed_placement_rejected():
         sfs.features(sfs.Csr(A.m, A.n, h(A.rp).pin_memory(), h(A.col).pin_memory(), d(A.val)))
     with pytest.raises(sfs.SfsError):  # pageable host memory
         sfs.features(sfs.Csr(A.m, A.n, h(A.rp), h(A.col), h(A.val)))
+
+
+def test_subset_labelling_races_only_representatives():
+    """f2 end to end: one representative per cluster is raced, every other matrix
+    is featurised only; the predicted labels of the representatives are their own race labels when their
+    cluster holds no other representative; the f4 scores are within their ranges."""
+    from paper_conf_icppw_dhandhaniadpbl21_b200 import predictor as pr
+    rng = np.random.default_rng(9)
+    mats, hosts = [], []
+    for i in range(24):
+        cls = [sfsgen.BAND, sfsgen.UNIFORM, sfsgen.BLOCKDIAG, sfsgen.POWERLAW][i % 4]
+        pa = 0.8 if cls in (sfsgen.BAND, sfsgen.BLOCKDIAG) else (12.0 if cls == sfsgen.UNIFORM else 2.4)
+        A = sfsgen.generate(sfsgen.make_spec(cls, seed=100 + i, m=int(rng.integers(3000, 20000)), ia=6, pa=pa))
+        hosts.append(A)
+        mats.append(to_dev(A))
+    opts = sfs.default_opts(reps=20, warmup=2)
+    _, full = sfs.label_corpus(mats, opts)
+    r = pr.subset_labelling(mats, opts, nc=6, k=1, truth=full)
+    assert r["raced"] <= 6 and r["others_not_raced"]
+    assert len(r["pred"]) == 24 and all(0 <= p < 5 for p in r["pred"])
+    q = r["quality"]
+    assert 0 < q["GT"] <= 1.0 and q["CSR"] > 0 and 0 <= q["Threshold"] <= 24 and 0 <= q["accuracy"] <= 1
+    assert r["t_subset_race_s"] > 0 and r["t_features_s"] > 0

@@ -61,11 +61,14 @@ def main():
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
     import sfsgen
 
+    from bench import ClockSampler  # nvidia-smi clocks and throttle reasons during the measurement
     for name in args.matrix.split(","):
-        run_one(args, name, torch, sfs, sfsgen)
+        clk = ClockSampler(torch.cuda.current_device())
+        clk.start()
+        run_one(args, name, torch, sfs, sfsgen, clk)
 
 
-def run_one(args, matrix, torch, sfs, sfsgen):
+def run_one(args, matrix, torch, sfs, sfsgen, clk=None):
     A = make_matrix(matrix)
     x = sfsgen.vector(3, A.n, A.dtype)
     t = lambda a: torch.from_numpy(a).cuda()
@@ -129,6 +132,8 @@ def run_one(args, matrix, torch, sfs, sfsgen):
             res.update(cold_us=cold, cold_gbs=nbytes / cold / 1e3, cold_frac=nbytes / cold / 1e3 / peak)
         out["formats"][name] = res
         M.free()
+    out["clocks"] = clk.stop() if clk else None
+    out["env"] = {k: v for k, v in os.environ.items() if k.startswith("SFS_")}
     s = json.dumps(out)
     print(f"{matrix:14s} m={A.m} nnz={A.nnz} " + "  ".join(
         f"{k} {v['hot_us']:.1f}us {v['hot_gbs']:.0f}GB/s" for k, v in out["formats"].items() if isinstance(v, dict)))
