@@ -78,7 +78,8 @@ typedef struct {
   int32_t csr_variant;      /* CSR kernel the library picks for this matrix (Q17): 0 vector (CUSP
                                mapping), 1 merge path, 2 stream (warp per 32 rows), 3 tile
                                (nnz-balanced 256-entry chunks, rows rebuilt from row_ptr), 4 tile
-                               with rows from a row-start bitmap (no empty rows) */
+                               with rows from a row-start bitmap (no empty rows), 5 tile with a
+                               bitmap over the non-empty rows and a rank -> row map (empty rows) */
 } sfs_features_t;
 
 typedef struct sfs_matrix_ *sfs_matrix; /* opaque, library-owned */
@@ -109,7 +110,7 @@ typedef struct {
   int64_t fill_slack;    /* (1<<20) */
   double hyb_rel_speed;  /* Q6 HYB width rule (3.0) */
   int64_t hyb_breakeven; /* (4096) */
-  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream; 3 = tile; 4 = tile with row ids from a row-start bitmap (falls back to 3 when a row is empty) */
+  int32_t csr_variant;   /* -1 = pick by Q17; 0 = vector; 1 = merge; 2 = stream; 3 = tile; 4 = tile with row ids from a row-start bitmap (becomes 5 when a row is empty); 5 = tile with a bitmap over the non-empty rows + rank -> row map */
   int32_t use_graphs;    /* 1 = capture the `reps` launches in one CUDA graph (0: direct launches with PDL) */
   const uint32_t *race_mask; /* sfs_label_corpus only, nullable (HOST array of n): matrix i races the
                                 formats formats_mask & race_mask[i]; 0 = features only (no conversion,

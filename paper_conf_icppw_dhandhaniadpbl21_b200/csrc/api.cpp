@@ -188,7 +188,7 @@ static void finalize(long long m, long long n, long long z, const DevAggr& a, lo
   if (a.empty_rows * 256 > (long long)z) f->csr_variant = 1;
   else if (mx > 4 * avg + 32 || z >= (1LL << 20)) f->csr_variant = a.empty_rows == 0 ? 4 : 3;
   else f->csr_variant = 2;
-  if (o.csr_variant >= 0 && o.csr_variant <= 4) f->csr_variant = o.csr_variant;
+  if (o.csr_variant >= 0 && o.csr_variant <= 5) f->csr_variant = o.csr_variant;
 }
 
 static sfs_status check_csr(const sfs_csr* A) {
@@ -386,9 +386,9 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         A->work = own(csr_merge_work_bytes(m, z, d.dtype));
         if (!A->work) return bail(SFS_ERR_OOM, "csr merge carries");
         BAIL_CUDA(launch_csr_merge_prepare((const int*)A->ptr[0], m, z, A->work, s));
-      } else if ((A->variant == 3 || A->variant == 4) && z > 0) {
-        if (A->variant == 4 && f.nnz_min < 1) A->variant = 3;  // the row-start bitmap needs every row non-empty
-        const int bitmap = A->variant == 4;
+      } else if ((A->variant == 3 || A->variant == 4 || A->variant == 5) && z > 0) {
+        if (A->variant == 4 && f.nnz_min < 1) A->variant = 5;  // empty rows: bitmap over the non-empty rows + map
+        const int bitmap = A->variant == 4 ? 1 : (A->variant == 5 ? 2 : 0);
         A->work = own(csr_tile_work_bytes(m, z, bitmap));
         if (!A->work) return bail(SFS_ERR_OOM, "csr tile partition");
         BAIL_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, bitmap, s));

@@ -77,6 +77,8 @@ cudaError_t launch_hyb_coo(const int* rp, long long m, long long K, long long* o
 size_t scan_work_bytes(long long m);
 cudaError_t launch_overflow_scan(const int* rp, long long m, int K, int* out, void* work, cudaStream_t s);
 cudaError_t launch_popc_scan(const unsigned* words, long long nw, int* out, void* work, cudaStream_t s);
+// pos[r] = number of non-empty rows before r (out[m] = non-empty rows): the CSR tile kernel's row map
+cudaError_t launch_nonempty_scan(const int* rp, long long m, int* out, void* work, cudaStream_t s);
 
 // ---------------------------------------------------------------- conversions (convert.cu)
 cudaError_t launch_csr2coo(int dtype, const int* rp, const int* col, const void* val, long long m, long long z,
@@ -131,7 +133,8 @@ struct Matrix {
   void* owned[8] = {nullptr};  // buffers to free
   int n_owned = 0;
   long long bytes = 0;
-  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile, 4 tile + row-start bitmap;
+  int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile, 4 tile + row-start bitmap,
+                               // 5 tile + bitmap over the non-empty rows + row map;
                                // HYB: 1 = one launch (ptr[5] = ovf)
   void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;

@@ -20,6 +20,10 @@ struct OverflowOp {
     return len > K ? len - K : 0;
   }
 };
+struct NonEmptyOp {
+  const int* rp;
+  __device__ __forceinline__ int operator()(long long i) const { return rp[i + 1] > rp[i] ? 1 : 0; }
+};
 struct PopcOp {
   const unsigned* w;
   __device__ __forceinline__ int operator()(long long i) const { return __popc(w[i]); }
@@ -120,6 +124,10 @@ size_t scan_work_bytes(long long n) { return sizeof(int) * (size_t)(ceil_div(n, 
 
 cudaError_t launch_overflow_scan(const int* rp, long long m, int K, int* out, void* work, cudaStream_t s) {
   return run_scan(OverflowOp{rp, K}, m, out, work, s);
+}
+
+cudaError_t launch_nonempty_scan(const int* rp, long long m, int* out, void* work, cudaStream_t s) {
+  return run_scan(NonEmptyOp{rp}, m, out, work, s);
 }
 
 cudaError_t launch_popc_scan(const unsigned* words, long long nw, int* out, void* work, cudaStream_t s) {

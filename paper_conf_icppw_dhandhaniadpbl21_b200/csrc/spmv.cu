@@ -621,12 +621,19 @@ __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, lo
 // built with the handle (bit k set iff entry k starts a row, z/8 bytes): lane l's 8 entries are byte l
 // of the chunk's 32-byte bitmap, row = a - 1 + (row starts up to the entry), a warp scan of the bytes'
 // popcounts -- no row_ptr loads and no shared-memory marks on the chunk's critical path.
-template <typename T, bool VEC, bool BM = false>
+//
+// MAP (variant 5, matrices with empty rows): the bitmap marks the starts of the NON-EMPTY rows only, row
+// ids are ranks among the non-empty rows (ca / srow converted to that numbering at handle creation) and
+// ne[j] maps rank j to its row; y was zeroed whole ahead of this grid (the empty rows stay 0), so no
+// per-chunk row_ptr walk is needed (variant 3's walk over runs of empty rows made it 3x slower than the
+// merge path on R-MAT).
+template <typename T, bool VEC, bool BM = false, bool MAP = false>
 __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const int* __restrict__ col,
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
                                               const int* __restrict__ ca, const int* __restrict__ srow,
-                                              long long nwarps, int* head, const unsigned* __restrict__ bm, int pf) {
+                                              long long nwarps, int* head, const unsigned* __restrict__ bm, int pf,
+                                              const int* __restrict__ ne) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
   const long long cb = warp * cpw;
@@ -634,13 +641,14 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
   const int own_lo = __ldg(ca + cb);  // rows >= own_lo start inside this range
   // the row split at the boundary with the next range (m: none); srow[w] rows were zeroed by
   // k_zero_rows before this grid touched y, and every piece of them is added atomically
-  const int next_split = warp + 1 < nwarps ? __ldg(srow + warp + 1) : (int)m;
+  const int next_split = warp + 1 < nwarps ? __ldg(srow + warp + 1) : (MAP ? 0x7fffffff : (int)m);
   int open_row = -1;                  // row left open at the previous chunk's end (all lanes agree)
   acc_t open = 0;
   bool waited = false;                // PDL: loads of the first chunk overlap k_zero_rows
+  auto yrow = [&](int row) -> int { return MAP ? __ldg(ne + row) : row; };
   auto emit = [&](int row, acc_t v) {
-    if (row < own_lo) atomicAdd(y + row, (T)v);  // the piece of the row carried into this range
-    else y[row] = (T)v;
+    if (row < own_lo) atomicAdd(y + yrow(row), (T)v);  // the piece of the row carried into this range
+    else y[yrow(row)] = (T)v;
   };
   int a_run = own_lo;  // BM: first row starting at or after the chunk start
   for (long long ch = cb; ch < ce; ch++) {
@@ -775,24 +783,25 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     open = __shfl_sync(0xffffffffu, S, 31);
   }
   if (l == 0 && open_row >= 0) {  // a piece of a split row if it continues past the range
-    if (open_row == next_split) atomicAdd(y + open_row, (T)open);
+    if (open_row == next_split) atomicAdd(y + yrow(open_row), (T)open);
     else emit(open_row, open);
   }
 }
 
 // blockDim is 64, 128 or 256 (smaller CTAs spread a small matrix's few warps over more SMs)
-template <typename T, bool VEC, bool BM>
+template <typename T, bool VEC, bool BM, bool MAP = false>
 __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
                                                                const int* __restrict__ ca, const int* __restrict__ srow,
-                                                               const unsigned* __restrict__ bm, int pf) {
+                                                               const unsigned* __restrict__ bm, int pf,
+                                                               const int* __restrict__ ne) {
   __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (warp < nwarps)
-    csr_tile_warp<T, VEC, BM>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps, s_head[BM ? 0 : threadIdx.x >> 5],
-                              bm, pf);
+    csr_tile_warp<T, VEC, BM, MAP>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps,
+                                   s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne);
   else
     pdl_wait();
   pdl_trigger();
@@ -826,11 +835,26 @@ __global__ void k_tile_split_rows(const int* __restrict__ rp, long long m, long 
   }
 }
 
-// row-start bitmap of a CSR without empty rows: bit k set iff entry k is the first of its row
-__global__ void k_row_starts(const int* __restrict__ rp, long long m, unsigned* __restrict__ bm) {
+// row-start bitmap: bit k set iff entry k is the first of its row (non-empty rows only: an empty row
+// has no entry; variant 4 has none, variant 5 maps ranks back with ne[]).  MAP: ne[pos[r]] = r.
+__global__ void k_row_starts(const int* __restrict__ rp, long long m, unsigned* __restrict__ bm,
+                             const int* __restrict__ pos, int* __restrict__ ne) {
   for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (long long)gridDim.x * blockDim.x) {
     const int k = __ldg(rp + r);
-    atomicOr(bm + (k >> 5), 1u << (k & 31));
+    if (__ldg(rp + r + 1) > k) {
+      atomicOr(bm + (k >> 5), 1u << (k & 31));
+      if (ne) ne[pos[r]] = (int)r;
+    }
+  }
+}
+
+// variant 5: chunk starts and split rows renumbered to ranks among the non-empty rows
+__global__ void k_tile_rank(const int* __restrict__ pos, long long m, int* __restrict__ a, long long nchunks,
+                            int* __restrict__ srow, long long nwarps) {
+  for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i <= nchunks || i < nwarps;
+       i += (long long)gridDim.x * blockDim.x) {
+    if (i <= nchunks) a[i] = pos[a[i]];  // a[i] <= m; pos[m] = number of non-empty rows
+    if (i < nwarps) srow[i] = srow[i] < m ? pos[srow[i]] : 0x7fffffff;
   }
 }
 
@@ -1445,7 +1469,8 @@ MergeWork merge_work(void* base, long long tiles) {
 struct TileWork {
   int* a;        // a_c = lower_bound(rp, 256 c), c = 0..nchunks
   int* srow;     // row split at the start of each warp range (m: none)
-  unsigned* bm;  // variant 4: row-start bitmap, nchunks * 8 words
+  unsigned* bm;  // variants 4, 5: row-start bitmap, nchunks * 8 words
+  int* ne;       // variant 5: row of each non-empty-row rank (m entries reserved)
 };
 TileWork tile_work(void* base, const TileGeom& g) {
   TileWork w;
@@ -1455,6 +1480,8 @@ TileWork tile_work(void* base, const TileGeom& g) {
   w.srow = (int*)p;
   p += al256(sizeof(int) * g.nwarps);
   w.bm = (unsigned*)p;
+  p += al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32));
+  w.ne = (int*)p;
   return w;
 }
 
@@ -1600,7 +1627,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       const int* rp = (const int*)A->ptr[0];
       const int* col = (const int*)A->ptr[1];
       const T* val = (const T*)A->ptr[2];
-      if (A->variant == 3 || A->variant == 4) {
+      if (A->variant == 3 || A->variant == 4 || A->variant == 5) {
         if (z == 0) {
           e = launch_zero<T>(y, m, s);
           break;
@@ -1624,8 +1651,14 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
         auto go = [&](auto kern) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
-                          (const int*)w.srow, (const unsigned*)w.bm, pf);
+                          (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne);
         };
+        if (A->variant == 5) {  // empty rows: all of y zeroed ahead (PDL-overlapped), ranks mapped to rows
+          e = launch_zero<T>(y, m, s);
+          if (e == cudaSuccess)
+            e = vec ? go(k_spmv_csr_tile<T, true, true, true>) : go(k_spmv_csr_tile<T, false, true, true>);
+          break;
+        }
         e = launch_k(k_zero_rows<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, y, (const int*)w.srow, g.nwarps, m);
         if (e == cudaSuccess) {
           if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>) : go(k_spmv_csr_tile<T, false, true>);
@@ -1723,11 +1756,13 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
   return cudaGetLastError();
 }
 
+// bitmap: 0 = variant 3, 1 = variant 4 (row-start bitmap), 2 = variant 5 (bitmap over the non-empty rows
+// + rank -> row map)
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
-  (void)m;
   const TileGeom g = tile_geom(z);
   return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) +
-         (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0);
+         (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0) +
+         (bitmap == 2 ? al256(sizeof(int) * m) : 0);
 }
 
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
@@ -1741,8 +1776,28 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
     cudaError_t e = cudaMemsetAsync(w.bm, 0, sizeof(unsigned) * g.nchunks * (kTChunk / 32), s);
     count_launch();
     if (e != cudaSuccess) return e;
-    k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm);
+    int* pos = nullptr;
+    void* sw = nullptr;
+    if (bitmap == 2) {  // ranks of the non-empty rows
+      pos = (int*)dalloc(sizeof(int) * (m + 1), s);
+      sw = dalloc(scan_work_bytes(m), s);
+      if (!pos || !sw) {
+        dfree(pos, s);
+        dfree(sw, s);
+        return cudaErrorMemoryAllocation;
+      }
+      e = launch_nonempty_scan(rp, m, pos, sw, s);
+      if (e != cudaSuccess) return e;
+    }
+    k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
     count_launch();
+    if (bitmap == 2) {
+      const long long items = std::max(g.nchunks + 1, g.nwarps);
+      k_tile_rank<<<grid_cap(items, 256, 8), 256, 0, s>>>(pos, m, w.a, g.nchunks, w.srow, g.nwarps);
+      count_launch();
+      dfree(pos, s);
+      dfree(sw, s);
+    }
   }
   return cudaGetLastError();
 }
@@ -1767,7 +1822,7 @@ int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) 
 
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
-    case SFS_CSR: return (A->variant == 1 || ((A->variant == 3 || A->variant == 4) && A->nnz > 0)) ? 2 : 1;
+    case SFS_CSR: return (A->variant == 1 || ((A->variant >= 3 && A->variant <= 5) && A->nnz > 0)) ? 2 : 1;
     case SFS_COO: return A->nnz > 0 ? 2 : 1;
     case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? 2 : 1;
     default: return 1;

@@ -38,6 +38,14 @@ def test_config2_rmat_22_fp32():
     fo = _full_check(A, formats=(sfs.CSR, sfs.COO, sfs.HYB), conv=True, ctx="configs[2]")
     assert not (fo["admissible_mask"] >> sfs.ELL) & 1 and not (fo["admissible_mask"] >> sfs.DIA) & 1
     assert fo["nnz"] > 60_000_000 and fo["nnz_max"] > 50_000
+    # every CSR kernel that handles empty rows, at full size (52 % of R-MAT's rows are empty)
+    dA = to_dev(A)
+    x = sfsgen.vector(2024, A.n, A.dtype)
+    for v in (1, 3, 5):
+        M = sfs.convert(dA, sfs.CSR, sfs.default_opts(csr_variant=v))
+        assert M.layout().variant == v
+        check_spmv(A, sfs.CSR, M, x, A.dtype, ctx=f"configs[2] CSR variant {v}")
+        M.free()
 
 
 def test_config3_stencil3d27_128_fp64():
@@ -67,9 +75,10 @@ def test_config4_corpus2000_largest_sample():
     _full_check(A, conv=False, ctx="corpus2000[164]")
 
 
-# fp32 DIA at bandwidth-bound sizes takes the TMA-staged kernel (k_spmv_dia_tma: >= 148*2*1024 rows):
-# the configs[3] stencil in fp32, a ragged stencil (343000 rows: partial last 1024-row block) and a
-# ragged 1M-row band, all formats, element by element against the oracle.
+# fp32 DIA at bandwidth-bound sizes (S = 1 launches of the consecutive-row kernels, k_spmv_dia_v4 and the
+# cp.async-staged k_spmv_dia_cpa when enabled): the configs[3] stencil in fp32, a ragged stencil (343000
+# rows: partial last 1024-row block) and a ragged 1M-row band, all formats, element by element against
+# the oracle.
 def test_config3_stencil3d27_128_fp32():
     A = sfsgen.stencil3d27(128, dtype=sfsgen.F32)
     fo = _full_check(A, formats=(sfs.ELL, sfs.DIA), conv=True, ctx="configs[3] fp32")

@@ -75,7 +75,7 @@ def test_conversions_bit_exact(name):
 
 
 @pytest.mark.parametrize("name", NAMES)
-@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4])
+@pytest.mark.parametrize("variant", [0, 1, 2, 3, 4, 5])
 def test_spmv_tolerance(name, variant):
     A = cases()[name]
     fo = oracle.features(A.m, A.n, A.rp, A.col)
@@ -353,7 +353,7 @@ def test_split_rows_and_gaps(shape):
     x = sfsgen.vector(3, n, A.dtype)
     dA = to_dev(A)
     for fmt, opts in [(sfs.CSR, sfs.default_opts(csr_variant=3)), (sfs.CSR, sfs.default_opts(csr_variant=1)),
-                      (sfs.COO, None)]:
+                      (sfs.CSR, sfs.default_opts(csr_variant=5)), (sfs.COO, None)]:
         M = sfs.convert(dA, fmt, opts)
         check_spmv(A, fmt, M, x, A.dtype, ctx=f"{shape}/{sfs.FORMAT_NAMES[fmt]}")
         M.free()
@@ -364,7 +364,7 @@ def test_split_rows_and_gaps(shape):
 def test_csr_bitmap_tile(dtype, cap):
     """CSR variant 4 (tile kernel with row ids from a row-start bitmap) on rows of 1..400,000 entries,
     rows of exactly 255/256/257/512, a row spanning many warp ranges; with empty rows present the
-    handle falls back to the row_ptr tile kernel (variant 3)."""
+    handle takes variant 5 (bitmap over the non-empty rows + rank -> row map, y zeroed ahead)."""
     A = _tile_edge_csr(dtype, cap, no_empty=True)
     x = sfsgen.vector(6, A.n, A.dtype)
     M = sfs.convert(to_dev(A), sfs.CSR, sfs.default_opts(csr_variant=4))
@@ -372,10 +372,12 @@ def test_csr_bitmap_tile(dtype, cap):
     check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="bitmap-tile")
     M.free()
     B = _tile_edge_csr(dtype, cap)
-    M = sfs.convert(to_dev(B), sfs.CSR, sfs.default_opts(csr_variant=4))
-    assert M.layout().variant == 3
-    check_spmv(B, sfs.CSR, M, x[:B.n] if len(x) >= B.n else sfsgen.vector(6, B.n, B.dtype), B.dtype, ctx="bitmap-fallback")
-    M.free()
+    for v in (4, 5):
+        M = sfs.convert(to_dev(B), sfs.CSR, sfs.default_opts(csr_variant=v))
+        assert M.layout().variant == 5
+        check_spmv(B, sfs.CSR, M, x[:B.n] if len(x) >= B.n else sfsgen.vector(6, B.n, B.dtype), B.dtype,
+                   ctx=f"bitmap-map/{v}")
+        M.free()
 
 
 @pytest.mark.parametrize("name", ["slack_at", "slack_past", "fill_at_dia", "fill_past_dia", "fill_at_ell",
