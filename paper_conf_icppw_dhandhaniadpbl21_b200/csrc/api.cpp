@@ -179,14 +179,14 @@ static void finalize(long long m, long long n, long long z, const DevAggr& a, lo
   if (f->ell_size <= lim) mask |= 1u << SFS_ELL;
   if (f->dia_size <= lim) mask |= 1u << SFS_DIA;
   f->admissible_mask = mask;
-  // Q17 (measured on corpus-200): merge path when empty rows are common (more than one
-  // per 256-entry chunk on average: a tile chunk would zero long runs of them, merge tiles count rows
-  // as work); else the tile kernel (nnz-balanced chunks) for skewed rows or nnz >= 2^20 -- with row
-  // ids from a row-start bitmap when no row is empty (variant 4), from row_ptr otherwise (3); else
-  // the stream kernel (warp per 32 rows), whose single launch is fastest on small regular matrices.
+  // Q17 (measured; profiles/r02/csr_variants.txt): matrices with empty rows take the tile
+  // kernel over the non-empty rows (variant 5: R-MAT 2^22 290 us against 336 for the merge path and
+  // 1020 for the row_ptr tile kernel); otherwise the tile kernel (nnz-balanced chunks, row ids from a
+  // row-start bitmap, variant 4) for skewed rows or nnz >= 2^20, else the stream kernel (warp per 32
+  // rows), whose single launch is fastest on small regular matrices.
   const long long avg = std::max(1LL, z / m);
-  if (a.empty_rows * 256 > (long long)z) f->csr_variant = 1;
-  else if (mx > 4 * avg + 32 || z >= (1LL << 20)) f->csr_variant = a.empty_rows == 0 ? 4 : 3;
+  if (a.empty_rows * 256 > (long long)z) f->csr_variant = 5;
+  else if (mx > 4 * avg + 32 || z >= (1LL << 20)) f->csr_variant = a.empty_rows == 0 ? 4 : 5;
   else f->csr_variant = 2;
   if (o.csr_variant >= 0 && o.csr_variant <= 5) f->csr_variant = o.csr_variant;
 }

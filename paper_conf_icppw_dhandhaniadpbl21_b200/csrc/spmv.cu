@@ -643,12 +643,14 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
   // k_zero_rows before this grid touched y, and every piece of them is added atomically
   const int next_split = warp + 1 < nwarps ? __ldg(srow + warp + 1) : (MAP ? 0x7fffffff : (int)m);
   int open_row = -1;                  // row left open at the previous chunk's end (all lanes agree)
+  int open_y = -1;                    // MAP: its y index
   acc_t open = 0;
   bool waited = false;                // PDL: loads of the first chunk overlap k_zero_rows
-  auto yrow = [&](int row) -> int { return MAP ? __ldg(ne + row) : row; };
-  auto emit = [&](int row, acc_t v) {
-    if (row < own_lo) atomicAdd(y + yrow(row), (T)v);  // the piece of the row carried into this range
-    else y[yrow(row)] = (T)v;
+  // emit(row, y index, value); MAP: the y index of a lane's first / last row is loaded as soon as the
+  // ranks are known (off the store path), rows strictly inside a lane's 8 entries (rare) load it there
+  auto emit = [&](int row, int yr, acc_t v) {
+    if (row < own_lo) atomicAdd(y + yr, (T)v);  // the piece of the row carried into this range
+    else y[yr] = (T)v;
   };
   int a_run = own_lo;  // BM: first row starting at or after the chunk start
   for (long long ch = cb; ch < ce; ch++) {
@@ -740,9 +742,10 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     // segmented reduction of (r[i], p[i]) exactly as in the COO kernel; padding items (past z) have
     // p = 0 and the last row
     const int rf = r[0], rl = r[kTV - 1];
+    const int yf = MAP ? __ldg(ne + (rf > 0 ? rf : 0)) : rf, yl = MAP ? __ldg(ne + (rl > 0 ? rl : 0)) : rl;
     const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
     if (open_row >= 0 && open_row != chunk_first) {
-      if (l == 0) emit(open_row, open);
+      if (l == 0) emit(open_row, MAP ? open_y : open_row, open);
       open_row = -1;
       open = 0;
     }
@@ -753,7 +756,7 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     for (int i = 1; i < kTV; i++) {
       if (r[i] != cr) {
         if (in_head) { hsum = cur; in_head = false; }
-        else emit(cr, cur);
+        else emit(cr, MAP ? __ldg(ne + cr) : cr, cur);
         cr = r[i];
         cur = p[i];
       } else {
@@ -777,14 +780,16 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     }
     const acc_t S_prev = __shfl_up_sync(0xffffffffu, S, 1);
     const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
-    if (!single) emit(rf, hsum + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0))));
-    if (l < 31 && next_rf != rl) emit(rl, S);
+    if (!single) emit(rf, yf, hsum + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0))));
+    if (l < 31 && next_rf != rl) emit(rl, yl, S);
     open_row = __shfl_sync(0xffffffffu, rl, 31);
+    if (MAP) open_y = __shfl_sync(0xffffffffu, yl, 31);
     open = __shfl_sync(0xffffffffu, S, 31);
   }
   if (l == 0 && open_row >= 0) {  // a piece of a split row if it continues past the range
-    if (open_row == next_split) atomicAdd(y + yrow(open_row), (T)open);
-    else emit(open_row, open);
+    const int oy = MAP ? open_y : open_row;
+    if (open_row == next_split) atomicAdd(y + oy, (T)open);
+    else emit(open_row, oy, open);
   }
 }
 
@@ -1213,12 +1218,19 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 // (the ELL mapping; warp = 128 consecutive rows, 512 contiguous bytes per slab load) and its 4 x values
 // are 4 scalar loads hitting the same lines (L1).  fp32's scalar strided mapping above moves 4 bytes
 // per load instruction; this one moves 16.  S diagonal-parts per row block meet in shared memory.
-template <typename T, int S, bool PUSH>
+//
+// XV (fp32, S <= 8, 16-byte aligned x): the 4 x values of a thread, x[r0+off .. r0+off+3], come from ONE
+// aligned 16-byte load at x[r0+off-s] (s = off mod 4, uniform over the warp since r0 is a multiple of 4)
+// plus the next thread's vector by warp shuffles (lane 31 loads its own), instead of 4 scalar loads
+// whose 16-byte lane stride spreads every warp instruction over 4-5 L1 wavefronts: x costs ~5
+// wavefronts per diagonal and warp instead of ~18.
+template <typename T, int S, bool PUSH, bool XV = false>
 __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __restrict__ offs,
                                                                 const T* __restrict__ dval,
                                                                 const T* __restrict__ x, T* __restrict__ y,
                                                                 long long m, long long n, long long P, int nd,
                                                                 PushParam<PUSH> push, int pfd) {
+  static_assert(!XV || (sizeof(T) == 4 && S <= 8), "XV: fp32, warps inside one diagonal part");
   constexpr int G = kDiaThreads / S;
   constexpr int kB = sizeof(T) == 4 ? 4 : 2;  // diagonals per batch (register cap)
   __shared__ int s_off[kDiaSmemOffs];
@@ -1249,7 +1261,46 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
         bool all_in = full && nb == kB;
 #pragma unroll
         for (int u = 0; u < kB; u++) all_in = all_in && r0 + off[u] >= 0 && r0 + off[u] + 3 < n;
-        if (all_in) {
+        bool warp_in = false;
+        if constexpr (XV) {
+          const bool full_warp = __activemask() == 0xffffffffu;
+          warp_in = full_warp && __all_sync(0xffffffffu, all_in);
+        }
+        if (warp_in) {
+          Vec4<T> v[kB];
+          T xv[kB][4];
+#pragma unroll
+          for (int u = 0; u < kB; u++) v[u].load_stream(dval + (long long)(d + u) * P + r0);
+          if (pfd > 0) {
+            const int dp = d + pfd * kB;
+#pragma unroll
+            for (int u = 0; u < kB; u++)
+              if (dp + u < d1)
+                asm volatile("prefetch.global.L2 [%0];" ::"l"(dval + (long long)(dp + u) * P + r0));
+          }
+          const int lane = threadIdx.x & 31;
+#pragma unroll
+          for (int u = 0; u < kB; u++) {
+            const long long base = r0 + off[u];
+            const int sft = (int)(base & 3);  // warp-uniform
+            const float4 a = __ldg(reinterpret_cast<const float4*>(x + (base - sft)));
+            float4 b;
+            b.x = __shfl_down_sync(0xffffffffu, a.x, 1);
+            b.y = __shfl_down_sync(0xffffffffu, a.y, 1);
+            b.z = __shfl_down_sync(0xffffffffu, a.z, 1);
+            if (lane == 31 && sft) b = __ldg(reinterpret_cast<const float4*>(x + (base - sft + 4)));
+            switch (sft) {
+              case 0: xv[u][0] = a.x; xv[u][1] = a.y; xv[u][2] = a.z; xv[u][3] = a.w; break;
+              case 1: xv[u][0] = a.y; xv[u][1] = a.z; xv[u][2] = a.w; xv[u][3] = b.x; break;
+              case 2: xv[u][0] = a.z; xv[u][1] = a.w; xv[u][2] = b.x; xv[u][3] = b.y; break;
+              default: xv[u][0] = a.w; xv[u][1] = b.x; xv[u][2] = b.y; xv[u][3] = b.z; break;
+            }
+          }
+#pragma unroll
+          for (int u = 0; u < kB; u++)
+#pragma unroll
+            for (int q = 0; q < 4; q++) acc[q] += (acc_t)v[u].v[q] * (acc_t)xv[u][q];
+        } else if (all_in) {
           Vec4<T> v[kB];
           T xv[kB][4];
 #pragma unroll
@@ -1543,12 +1594,21 @@ bool dia_v4_enabled(size_t elem) {
   return elem == 4 ? f32 : f64;
 }
 
+// fp32 consecutive-row DIA with aligned x vectors + shuffles (k_spmv_dia_v4<..., XV>); SFS_DIA_XV=0 disables
+bool dia_xv_enabled() {
+  static const bool v = [] {
+    const char* e = getenv("SFS_DIA_XV");
+    return !(e && e[0] == '0');
+  }();
+  return v;
+}
+
 // cp.async-staged DIA (k_spmv_dia_cpa) for S = 1 launches of at least SFS_DIA_CPA_ROWS rows (default
-// 2^18): fp32 by default; SFS_DIA_CPA=0 disables, SFS_DIA_CPA=2 also enables fp64 (A/B switches)
+// 2^18): SFS_DIA_CPA=1 enables it for fp32, 2 also for fp64 (A/B switches; off by default)
 bool dia_cpa_enabled(size_t elem, long long m) {
-  static const int mode = [] {
+  static const int mode = [] {  // default off: measured slower than k_spmv_dia_v4 (profiles/r02)
     const char* e = getenv("SFS_DIA_CPA");
-    return e ? atoi(e) : 1;
+    return e ? atoi(e) : 0;
   }();
   static const long long min_rows = [] {
     const char* e = getenv("SFS_DIA_CPA_ROWS");
@@ -1601,6 +1661,16 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
       return e ? atoi(e) : 1;
     }();
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
+    if constexpr (sizeof(T) == 4) {
+      if (dia_xv_enabled() && S <= 8 && ((uintptr_t)x % 16) == 0) {
+        switch (S) {
+          case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          case 4: return launch_k(k_spmv_dia_v4<T, 4, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          default: return launch_k(k_spmv_dia_v4<T, 8, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+        }
+      }
+    }
     switch (S) {
       case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
       case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);

@@ -39,6 +39,8 @@ def make_matrix(name):
         return sfsgen.generate(sfsgen.make_spec(sfsgen.BLOCKDIAG, seed=14, m=1_500_000, ia=40, pa=0.75))
     if name == "uniform_big":
         return sfsgen.generate(sfsgen.make_spec(sfsgen.UNIFORM, seed=12, m=1_000_000, pa=40.0))
+    if name == "band_big_f32":
+        return sfsgen.generate(sfsgen.make_spec(sfsgen.BAND, seed=11, m=1_000_000, ia=24, pa=0.8, dtype=sfsgen.F32))
     if name == "powerlaw_big":
         return sfsgen.generate(sfsgen.make_spec(sfsgen.POWERLAW, seed=13, m=2_000_000, pa=2.2, dtype=sfsgen.F32))
     raise ValueError(name)
