@@ -45,6 +45,16 @@ def build_gen(force=False):
     return out
 
 
+def build_gen_device(force=False):
+    """sfsgen/libsfsgen_dev.so: the generators on the GPU (CUB sorts), bit-identical to gen.c."""
+    src = [os.path.join(ROOT, "sfsgen", "gen_device.cu"), os.path.join(ROOT, "sfsgen", "sfsgen.h")]
+    out = os.path.join(ROOT, "sfsgen", "libsfsgen_dev.so")
+    if force or _stale(out, src):
+        _run([NVCC, "-O3", "-std=c++17", "-shared", "-Xcompiler", "-fPIC,-ffp-contract=off", "-lineinfo"] + ARCH +
+             ["-I", os.path.join(ROOT, "sfsgen"), src[0], "-o", out, "-cudart", "static"])
+    return out
+
+
 def build_oracle(force=False):
     src = [os.path.join(ROOT, "oracle", f) for f in ("oracle.c", "semisup.c", "oracle.h")]
     out = os.path.join(ROOT, "oracle", "liboracle.so")
@@ -85,6 +95,7 @@ def build_sfs(force=False, verbose=False, variant="", defines=()):
 
 def build_all(force=False):
     build_gen(force)
+    build_gen_device(force)
     build_oracle(force)
     if glob.glob(os.path.join(CSRC, "*.cu")):
         build_sfs(force)

@@ -31,7 +31,6 @@
 #include <stdlib.h>
 
 #include <algorithm>
-#include <mutex>
 
 #include "common.cuh"
 #include "internal.h"
@@ -63,21 +62,6 @@ bool pdl_enabled() {
 }
 
 // cudaLaunchKernelEx with the programmatic-stream-serialization attribute (PDL).
-template <typename... Params, typename... Args>
-cudaError_t launch_kx(void (*kern)(Params...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
-  cfg.blockDim = block;
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = s;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  count_launch();
-  return cudaLaunchKernelEx(&cfg, kern, static_cast<Params>(args)...);
-}
 template <typename... Params, typename... Args>
 cudaError_t launch_k(void (*kern)(Params...), dim3 grid, dim3 block, cudaStream_t s, Args... args) {
   cudaLaunchConfig_t cfg = {};
@@ -1218,19 +1202,12 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 // (the ELL mapping; warp = 128 consecutive rows, 512 contiguous bytes per slab load) and its 4 x values
 // are 4 scalar loads hitting the same lines (L1).  fp32's scalar strided mapping above moves 4 bytes
 // per load instruction; this one moves 16.  S diagonal-parts per row block meet in shared memory.
-//
-// XV (fp32, S <= 8, 16-byte aligned x): the 4 x values of a thread, x[r0+off .. r0+off+3], come from ONE
-// aligned 16-byte load at x[r0+off-s] (s = off mod 4, uniform over the warp since r0 is a multiple of 4)
-// plus the next thread's vector by warp shuffles (lane 31 loads its own), instead of 4 scalar loads
-// whose 16-byte lane stride spreads every warp instruction over 4-5 L1 wavefronts: x costs ~5
-// wavefronts per diagonal and warp instead of ~18.
-template <typename T, int S, bool PUSH, bool XV = false>
+template <typename T, int S, bool PUSH>
 __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __restrict__ offs,
                                                                 const T* __restrict__ dval,
                                                                 const T* __restrict__ x, T* __restrict__ y,
                                                                 long long m, long long n, long long P, int nd,
                                                                 PushParam<PUSH> push, int pfd) {
-  static_assert(!XV || (sizeof(T) == 4 && S <= 8), "XV: fp32, warps inside one diagonal part");
   constexpr int G = kDiaThreads / S;
   constexpr int kB = sizeof(T) == 4 ? 4 : 2;  // diagonals per batch (register cap)
   __shared__ int s_off[kDiaSmemOffs];
@@ -1261,46 +1238,7 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
         bool all_in = full && nb == kB;
 #pragma unroll
         for (int u = 0; u < kB; u++) all_in = all_in && r0 + off[u] >= 0 && r0 + off[u] + 3 < n;
-        bool warp_in = false;
-        if constexpr (XV) {
-          const bool full_warp = __activemask() == 0xffffffffu;
-          warp_in = full_warp && __all_sync(0xffffffffu, all_in);
-        }
-        if (warp_in) {
-          Vec4<T> v[kB];
-          T xv[kB][4];
-#pragma unroll
-          for (int u = 0; u < kB; u++) v[u].load_stream(dval + (long long)(d + u) * P + r0);
-          if (pfd > 0) {
-            const int dp = d + pfd * kB;
-#pragma unroll
-            for (int u = 0; u < kB; u++)
-              if (dp + u < d1)
-                asm volatile("prefetch.global.L2 [%0];" ::"l"(dval + (long long)(dp + u) * P + r0));
-          }
-          const int lane = threadIdx.x & 31;
-#pragma unroll
-          for (int u = 0; u < kB; u++) {
-            const long long base = r0 + off[u];
-            const int sft = (int)(base & 3);  // warp-uniform
-            const float4 a = __ldg(reinterpret_cast<const float4*>(x + (base - sft)));
-            float4 b;
-            b.x = __shfl_down_sync(0xffffffffu, a.x, 1);
-            b.y = __shfl_down_sync(0xffffffffu, a.y, 1);
-            b.z = __shfl_down_sync(0xffffffffu, a.z, 1);
-            if (lane == 31 && sft) b = __ldg(reinterpret_cast<const float4*>(x + (base - sft + 4)));
-            switch (sft) {
-              case 0: xv[u][0] = a.x; xv[u][1] = a.y; xv[u][2] = a.z; xv[u][3] = a.w; break;
-              case 1: xv[u][0] = a.y; xv[u][1] = a.z; xv[u][2] = a.w; xv[u][3] = b.x; break;
-              case 2: xv[u][0] = a.z; xv[u][1] = a.w; xv[u][2] = b.x; xv[u][3] = b.y; break;
-              default: xv[u][0] = a.w; xv[u][1] = b.x; xv[u][2] = b.y; xv[u][3] = b.z; break;
-            }
-          }
-#pragma unroll
-          for (int u = 0; u < kB; u++)
-#pragma unroll
-            for (int q = 0; q < 4; q++) acc[q] += (acc_t)v[u].v[q] * (acc_t)xv[u][q];
-        } else if (all_in) {
+        if (all_in) {
           Vec4<T> v[kB];
           T xv[kB][4];
 #pragma unroll
@@ -1354,148 +1292,6 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
         if (r0 + q < m) store_row<PUSH>(y, r0 + q, (T)acc[q], push, pushed);
     }
   }
-  halo_signal<PUSH>(push, pushed);
-  pdl_trigger();
-}
-
-// Streaming DIA with the slab staged by cp.async (LDGSTS, L2 -> shared, no registers held): thread = 4
-// consecutive rows (the v4 mapping), block = 1024 rows, every diagonal of the block in batches of 4.
-// Each thread runs its own software pipeline over its flattened (block, batch) sequence: the slab
-// vectors of the batch kCpaStages - 1 ahead are in flight as cp.async copies into the thread's own
-// slice of a shared-memory ring while the current batch's x gathers and FMAs run, so HBM sees
-// kCpaStages x 4 x 16 B per thread in flight without a register cost (the v4 kernel holds one batch in
-// registers and relies on an L2 prefetch).  A thread only reads the ring slots it filled, so
-// cp.async.wait_group is the only synchronisation.  S = 1 (bandwidth-bound sizes).
-constexpr int kCpaStages = 4;
-constexpr int kCpaBatch = 4;
-template <typename T> constexpr int cpa_vecs() { return (int)(4 * sizeof(T) / 16); }  // 16-byte copies per diagonal
-template <typename T> constexpr size_t cpa_smem() {
-  return (size_t)kCpaStages * kCpaBatch * cpa_vecs<T>() * kDiaThreads * 16;
-}
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-  const unsigned sa = (unsigned)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(sa), "l"(gmem) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
-
-template <typename T, bool PUSH>
-__global__ void __launch_bounds__(kDiaThreads, 3) k_spmv_dia_cpa(const int* __restrict__ offs,
-                                                                 const T* __restrict__ dval,
-                                                                 const T* __restrict__ x, T* __restrict__ y,
-                                                                 long long m, long long n, long long P, int nd,
-                                                                 PushParam<PUSH> push) {
-  constexpr int kB = kCpaBatch, NS = kCpaStages, VPD = cpa_vecs<T>();
-  constexpr long long kRowsBlk = (long long)kDiaThreads * 4;
-  extern __shared__ uint4 s_ring[];  // [NS][kB][VPD][kDiaThreads]
-  __shared__ int s_off[kDiaSmemOffs];
-  pdl_wait();
-  pdl_early();
-  const int tid = threadIdx.x;
-  const long long nblk = ceil_div(m, kRowsBlk);
-  const int nbat = (nd + kB - 1) / kB;
-  const long long myblk = (long long)blockIdx.x < nblk ? ceil_div(nblk - blockIdx.x, (long long)gridDim.x) : 0;
-  const long long nitems = myblk * nbat;
-  // the slab does not depend on x: the first stages are issued before the x-side waits.  Producer and
-  // consumer walk the same (block, batch) sequence with their own counters (no 64-bit divisions).
-  const long long rstride = (long long)gridDim.x * kRowsBlk;
-  long long i_r0 = (long long)blockIdx.x * kRowsBlk + 4 * tid;  // producer position
-  int i_d = 0, i_slot = 0;
-  long long left = nitems;
-  auto issue = [&]() {
-    if (left > 0) {
-      if (i_r0 < m) {
-#pragma unroll
-        for (int u = 0; u < kB; u++)
-          if (i_d + u < nd) {
-            const T* src = dval + (long long)(i_d + u) * P + i_r0;
-#pragma unroll
-            for (int v = 0; v < VPD; v++)
-              cp_async16(&s_ring[((i_slot * kB + u) * VPD + v) * kDiaThreads + tid], src + v * (16 / sizeof(T)));
-          }
-      }
-      left--;
-      i_d += kB;
-      if (i_d >= nd) {
-        i_d = 0;
-        i_r0 += rstride;
-      }
-      i_slot = i_slot + 1 == NS ? 0 : i_slot + 1;
-    }
-    cp_async_commit();
-  };
-#pragma unroll
-  for (int i = 0; i < NS - 1; i++) issue();
-  const int nsm = nd < kDiaSmemOffs ? nd : kDiaSmemOffs;
-  for (int i = tid; i < nsm; i += blockDim.x) s_off[i] = offs[i];
-  __syncthreads();
-  halo_wait<PUSH>(push);
-  bool pushed = false;
-  acc_t acc[4] = {0, 0, 0, 0};
-  long long r0 = (long long)blockIdx.x * kRowsBlk + 4 * tid;  // consumer position
-  int d = 0, slot = 0;
-  for (long long it = 0; it < nitems; it++) {
-    issue();
-    const bool live = r0 < m;
-    const int nb = nd - d < kB ? nd - d : kB;
-    int off[kB];
-#pragma unroll
-    for (int u = 0; u < kB; u++) off[u] = u < nb ? (d + u < kDiaSmemOffs ? s_off[d + u] : __ldg(offs + d + u)) : 0;
-    bool all_in = live && r0 + 4 <= m && nb == kB;
-#pragma unroll
-    for (int u = 0; u < kB; u++) all_in = all_in && r0 + off[u] >= 0 && r0 + off[u] + 3 < n;
-    T xv[kB][4];
-    if (all_in) {  // x gathers issued before waiting on the slab copies
-#pragma unroll
-      for (int u = 0; u < kB; u++) {
-        const T* xp = x + r0 + off[u];
-#pragma unroll
-        for (int q = 0; q < 4; q++) xv[u][q] = ld_x(xp + q);
-      }
-    }
-    cp_async_wait<NS - 1>();  // this thread's copies of this batch have landed
-    if (live) {
-#pragma unroll
-      for (int u = 0; u < kB; u++) {
-        if (u < nb) {
-          T v[4];
-#pragma unroll
-          for (int w = 0; w < VPD; w++) {
-            const uint4 q4 = s_ring[((slot * kB + u) * VPD + w) * kDiaThreads + tid];
-            const T* pv = reinterpret_cast<const T*>(&q4);
-#pragma unroll
-            for (int e = 0; e < (int)(16 / sizeof(T)); e++) v[w * (16 / sizeof(T)) + e] = pv[e];
-          }
-          if (all_in) {
-#pragma unroll
-            for (int q = 0; q < 4; q++) acc[q] += (acc_t)v[q] * (acc_t)xv[u][q];
-          } else {
-#pragma unroll
-            for (int q = 0; q < 4; q++) {
-              const long long c = r0 + q + off[u];
-              if (r0 + q < m && c >= 0 && c < n) acc[q] += (acc_t)v[q] * (acc_t)ld_x(x + c);
-            }
-          }
-        }
-      }
-    }
-    slot = slot + 1 == NS ? 0 : slot + 1;
-    d += kB;
-    if (d >= nd) {  // last batch of this block: the rows are complete
-      if (live) {
-#pragma unroll
-        for (int q = 0; q < 4; q++)
-          if (r0 + q < m) store_row<PUSH>(y, r0 + q, (T)acc[q], push, pushed);
-      }
-#pragma unroll
-      for (int q = 0; q < 4; q++) acc[q] = 0;
-      d = 0;
-      r0 += rstride;
-    }
-  }
-  cp_async_wait<0>();
   halo_signal<PUSH>(push, pushed);
   pdl_trigger();
 }
@@ -1594,30 +1390,6 @@ bool dia_v4_enabled(size_t elem) {
   return elem == 4 ? f32 : f64;
 }
 
-// fp32 consecutive-row DIA with aligned x vectors + shuffles (k_spmv_dia_v4<..., XV>); SFS_DIA_XV=0 disables
-bool dia_xv_enabled() {
-  static const bool v = [] {
-    const char* e = getenv("SFS_DIA_XV");
-    return !(e && e[0] == '0');
-  }();
-  return v;
-}
-
-// cp.async-staged DIA (k_spmv_dia_cpa) for S = 1 launches of at least SFS_DIA_CPA_ROWS rows (default
-// 2^18): SFS_DIA_CPA=1 enables it for fp32, 2 also for fp64 (A/B switches; off by default)
-bool dia_cpa_enabled(size_t elem, long long m) {
-  static const int mode = [] {  // default off: measured slower than k_spmv_dia_v4 (profiles/r02)
-    const char* e = getenv("SFS_DIA_CPA");
-    return e ? atoi(e) : 0;
-  }();
-  static const long long min_rows = [] {
-    const char* e = getenv("SFS_DIA_CPA_ROWS");
-    return e ? atoll(e) : (1LL << 18);
-  }();
-  if (m < min_rows || mode == 0) return false;
-  return elem == 4 ? true : mode == 2;
-}
-
 template <typename T, bool PUSH>
 cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushParam<PUSH> push) {
   const long long m = A->m;
@@ -1639,20 +1411,6 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   const int* offs = (const int*)A->ptr[0];
   const T* dv = (const T*)A->ptr[1];
   const int nd = (int)A->ndiag;
-  if (S == 1 && nd > 0 && dia_cpa_enabled(sizeof(T), m)) {
-    // cp.async-staged slab (bandwidth-bound sizes); CTAs of 1024 rows, blocks balanced over the CTAs
-    const long long nb = ceil_div(m, (long long)kDiaThreads * 4), cap = (long long)kSMs * 3;
-    const long long per = ceil_div(nb, cap);
-    const int g = (int)ceil_div(nb, per);
-    static std::once_flag once[kMaxDevices];
-    int dev = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
-    std::call_once(once[dev], [] {
-      cudaFuncSetAttribute(k_spmv_dia_cpa<T, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cpa_smem<T>());
-      cudaFuncSetAttribute(k_spmv_dia_cpa<T, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)cpa_smem<T>());
-    });
-    return launch_kx(k_spmv_dia_cpa<T, PUSH>, dim3(g), bd, cpa_smem<T>(), s, offs, dv, x, y, m, A->n, A->pitch, nd, push);
-  }
   if (dia_v4_enabled(sizeof(T))) {
     // L2 prefetch of the next batch's slab (SFS_DIA_PF: distance in batches, 0 = off; A/B switch).
     // 128^3 fp32 stencil cold (tools/ab_dia_pf.sh): off 54.3 us (0.69), 1: 52.2 us (0.71), 2: 53.2, 3: 55.3
@@ -1661,16 +1419,6 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
       return e ? atoi(e) : 1;
     }();
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
-    if constexpr (sizeof(T) == 4) {
-      if (dia_xv_enabled() && S <= 8 && ((uintptr_t)x % 16) == 0) {
-        switch (S) {
-          case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
-          case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
-          case 4: return launch_k(k_spmv_dia_v4<T, 4, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
-          default: return launch_k(k_spmv_dia_v4<T, 8, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
-        }
-      }
-    }
     switch (S) {
       case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
       case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);

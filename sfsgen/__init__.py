@@ -158,3 +158,63 @@ def from_dense(a: np.ndarray, dtype=None) -> CSR:
                 vals.append(a[r, c])
         rp.append(len(cols))
     return CSR(m, n, np.array(rp, np.int32), np.array(cols, np.int32), np.array(vals, dtype))
+
+
+# ---------------------------------------------------------------- the same generators on the GPU
+# libsfsgen_dev.so (gen_device.cu): bit-identical CSR built in device memory (§8(d) C5
+# "Generated on device per rank").  Returned as torch tensors on the current CUDA device.
+DEV_LIB_PATH = os.path.join(_HERE, "libsfsgen_dev.so")
+_dlib = None
+
+
+def dlib():
+    global _dlib
+    if _dlib is None:
+        if not os.path.exists(DEV_LIB_PATH):
+            raise RuntimeError(f"{DEV_LIB_PATH} missing: run build_native.build_gen_device()")
+        L = ctypes.CDLL(DEV_LIB_PATH)
+        L.sfsgen_generate_device.argtypes = [ctypes.POINTER(Spec), ctypes.POINTER(_CSR), ctypes.c_void_p]
+        L.sfsgen_generate_device.restype = ctypes.c_int
+        L.sfsgen_free_device.argtypes = [ctypes.POINTER(_CSR)]
+        L.sfsgen_vector_device.argtypes = [ctypes.c_uint64, ctypes.c_int64, ctypes.c_int32, ctypes.c_void_p,
+                                           ctypes.c_void_p]
+        L.sfsgen_vector_device.restype = ctypes.c_int
+        _dlib = L
+    return _dlib
+
+
+class _DevBuf:
+    def __init__(self, ptr, n, typestr):
+        self.__cuda_array_interface__ = {"shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 3,
+                                         "strides": None}
+
+
+def generate_device(spec: Spec):
+    """(m, n, rp, col, val) with rp/col/val torch tensors on the current CUDA device (copies of the library's
+    buffers, which are freed before returning)."""
+    import torch
+    out = _CSR()
+    st = torch.cuda.current_stream()
+    rc = dlib().sfsgen_generate_device(ctypes.byref(spec), ctypes.byref(out), st.cuda_stream)
+    if rc != 0:
+        raise RuntimeError(f"sfsgen_generate_device failed for {spec.describe()}")
+    try:
+        m, nnz = int(out.m), int(out.nnz)
+        dev = torch.device("cuda", torch.cuda.current_device())
+        view = lambda p, k, t: torch.as_tensor(_DevBuf(ctypes.cast(p, ctypes.c_void_p).value, k, t), device=dev)
+        rp = view(out.rp, m + 1, "<i4").clone()
+        col = view(out.col, max(nnz, 1), "<i4")[:nnz].clone()
+        val = view(out.val, max(nnz, 1), "<f8" if out.dtype else "<f4")[:nnz].clone()
+        torch.cuda.synchronize()
+        return m, int(out.n), rp, col, val
+    finally:
+        dlib().sfsgen_free_device(ctypes.byref(out))
+
+
+def vector_device(seed: int, n: int, dtype: int = F64):
+    import torch
+    x = torch.empty(n, dtype=torch.float64 if dtype else torch.float32, device="cuda")
+    if dlib().sfsgen_vector_device(seed & 0xFFFFFFFFFFFFFFFF, n, dtype, x.data_ptr(),
+                                   torch.cuda.current_stream().cuda_stream) != 0:
+        raise RuntimeError("sfsgen_vector_device failed")
+    return x

@@ -63,6 +63,14 @@ int sfsgen_corpus_spec(int32_t corpus, int64_t i, sfsgen_spec *out);
 /* Number of threads the generator uses (OpenMP). */
 int sfsgen_threads(void);
 
+/* The same generators on the GPU (gen_device.cu, libsfsgen_dev.so): bit-identical CSR in device memory
+   (cudaMalloc'd rp/col/val; free with sfsgen_free_device), stream-ordered on `stream` (a cudaStream_t),
+   synchronizes it before returning.  Returns 0 on success. */
+int sfsgen_generate_device(const sfsgen_spec *s, sfsgen_csr *out, void *stream);
+void sfsgen_free_device(sfsgen_csr *c);
+/* x on the device (out: n entries of dtype), asynchronous on `stream`. */
+int sfsgen_vector_device(uint64_t seed, int64_t n, int32_t dtype, void *out, void *stream);
+
 #ifdef __cplusplus
 }
 #endif

@@ -65,13 +65,13 @@ def main():
 
     from bench import ClockSampler  # nvidia-smi clocks and throttle reasons during the measurement
     for name in args.matrix.split(","):
-        clk = ClockSampler(torch.cuda.current_device())
-        clk.start()
-        run_one(args, name, torch, sfs, sfsgen, clk)
+        run_one(args, name, torch, sfs, sfsgen, ClockSampler(torch.cuda.current_device()))
 
 
 def run_one(args, matrix, torch, sfs, sfsgen, clk=None):
     A = make_matrix(matrix)
+    if clk:  # sampled from here: the (host) generation above leaves the GPU idle at low clocks
+        clk.start()
     x = sfsgen.vector(3, A.n, A.dtype)
     t = lambda a: torch.from_numpy(a).cuda()
     dA = sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val))
