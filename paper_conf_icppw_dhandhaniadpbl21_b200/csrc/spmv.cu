@@ -553,6 +553,50 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
   pdl_trigger();
 }
 
+// Boundary records of the one-launch COO and CSR tile kernels (FIX): instead of atomically adding into
+// a y zeroed by a preceding kernel (the zero / zero-rows launch), warp w writes the piece of the row
+// split at its range start (F record) and its final carry (L record); rows inside a range are stored by
+// their warp.  The last CTA to finish (acq_rel ticket) sums the records of equal rows -- the sequence
+// F0 L0 F1 L1 ... is ordered by row -- stores them and resets the ticket for the next launch.  Valid
+// only when every row holds an entry (rows the kernel never sees would stay unwritten), which the
+// handle checks at conversion.
+struct CooFix {
+  int* rrow;        // 2 * nwarps
+  acc_t* rval;      // 2 * nwarps
+  unsigned* ticket; // 1
+};
+
+template <typename T, bool ACCUM>
+__device__ void coo_fixup(T* __restrict__ y, const CooFix& fx, long long nrec) {
+  for (long long i = threadIdx.x; i < nrec; i += blockDim.x) {
+    const int r = __ldcg(fx.rrow + i);
+    if (r < 0 || (i > 0 && __ldcg(fx.rrow + i - 1) == r)) continue;  // not the first record of its row
+    acc_t v = 0;
+    for (long long j = i; j < nrec && __ldcg(fx.rrow + j) == r; j++) v += __ldcg(fx.rval + j);
+    if (ACCUM) y[r] = (T)((acc_t)y[r] + v);
+    else y[r] = (T)v;
+  }
+}
+
+// Every thread of the grid calls this after its records are written (and fenced): the last CTA applies
+// them.
+template <typename T, bool ACCUM>
+__device__ __forceinline__ void fix_finish(T* __restrict__ y, const CooFix& fx, long long nrec) {
+  __shared__ bool s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned prev;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev) : "l"(fx.ticket) : "memory");
+    s_last = prev == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (s_last) {
+    __threadfence();
+    coo_fixup<T, ACCUM>(y, fx, nrec);
+    if (threadIdx.x == 0) *fx.ticket = 0u;
+  }
+}
+
 // ======================================================================== CSR tile (nnz-balanced)
 // The COO kernel's shape on the CSR arrays.  Warp w streams the contiguous chunks [cb, ce) of 256
 // entries (8 per lane, 256-bit col/val loads whose addresses do not depend on row_ptr), and the row of
@@ -611,13 +655,13 @@ __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, lo
 // ne[j] maps rank j to its row; y was zeroed whole ahead of this grid (the empty rows stay 0), so no
 // per-chunk row_ptr walk is needed (variant 3's walk over runs of empty rows made it 3x slower than the
 // merge path on R-MAT).
-template <typename T, bool VEC, bool BM = false, bool MAP = false>
+template <typename T, bool VEC, bool BM = false, bool MAP = false, bool FIX = false>
 __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const int* __restrict__ col,
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
                                               const int* __restrict__ ca, const int* __restrict__ srow,
                                               long long nwarps, int* head, const unsigned* __restrict__ bm, int pf,
-                                              const int* __restrict__ ne) {
+                                              const int* __restrict__ ne, const CooFix& fx) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
   const long long cb = warp * cpw;
@@ -632,9 +676,14 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
   bool waited = false;                // PDL: loads of the first chunk overlap k_zero_rows
   // emit(row, y index, value); MAP: the y index of a lane's first / last row is loaded as soon as the
   // ranks are known (off the store path), rows strictly inside a lane's 8 entries (rare) load it there
+  acc_t split_piece = 0;  // FIX: this lane's pieces of the row split at the range start (< own_lo)
   auto emit = [&](int row, int yr, acc_t v) {
-    if (row < own_lo) atomicAdd(y + yr, (T)v);  // the piece of the row carried into this range
-    else y[yr] = (T)v;
+    if (row < own_lo) {  // the piece of the row carried into this range
+      if (FIX) split_piece += v;
+      else atomicAdd(y + yr, (T)v);
+    } else {
+      y[yr] = (T)v;
+    }
   };
   int a_run = own_lo;  // BM: first row starting at or after the chunk start
   for (long long ch = cb; ch < ce; ch++) {
@@ -770,6 +819,21 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     if (MAP) open_y = __shfl_sync(0xffffffffu, yl, 31);
     open = __shfl_sync(0xffffffffu, S, 31);
   }
+  if constexpr (FIX) {
+    static_assert(!MAP, "records hold row ids");
+    const bool cont = open_row >= 0 && open_row == next_split;  // continues past the range (lane-uniform)
+    if (l == 0 && open_row >= 0 && !cont) emit(open_row, open_row, open);
+    split_piece = warp_sum(split_piece);
+    if (l == 0) {
+      const int sr = __ldg(srow + warp);  // the row split at this range's start (m: none)
+      fx.rrow[2 * warp] = sr < (int)m ? sr : -1;
+      fx.rval[2 * warp] = split_piece;
+      fx.rrow[2 * warp + 1] = cont ? open_row : -1;
+      fx.rval[2 * warp + 1] = cont ? open : acc_t(0);
+      __threadfence();
+    }
+    return;
+  }
   if (l == 0 && open_row >= 0) {  // a piece of a split row if it continues past the range
     const int oy = MAP ? open_y : open_row;
     if (open_row == next_split) atomicAdd(y + oy, (T)open);
@@ -778,21 +842,27 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
 }
 
 // blockDim is 64, 128 or 256 (smaller CTAs spread a small matrix's few warps over more SMs)
-template <typename T, bool VEC, bool BM, bool MAP = false>
+template <typename T, bool VEC, bool BM, bool MAP = false, bool FIX = false>
 __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
                                                                const int* __restrict__ ca, const int* __restrict__ srow,
                                                                const unsigned* __restrict__ bm, int pf,
-                                                               const int* __restrict__ ne) {
+                                                               const int* __restrict__ ne, CooFix fx) {
   __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (warp < nwarps)
-    csr_tile_warp<T, VEC, BM, MAP>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps,
-                                   s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne);
-  else
+  if (warp < nwarps) {
+    csr_tile_warp<T, VEC, BM, MAP, FIX>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps,
+                                        s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne, fx);
+  } else {
     pdl_wait();
+    if (FIX && (threadIdx.x & 31) == 0) {  // a warp past the last range: no records
+      fx.rrow[2 * warp] = fx.rrow[2 * warp + 1] = -1;
+      __threadfence();
+    }
+  }
+  if (FIX) fix_finish<T, false>(y, fx, 2 * (long long)gridDim.x * (blockDim.x >> 5));
   pdl_trigger();
 }
 
@@ -859,10 +929,11 @@ __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
   else y[row] = (T)v;
 }
 
-template <typename T, bool ACCUM>
+template <typename T, bool ACCUM, bool FIX = false>
 __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
-                                                          T* __restrict__ y, long long z, long long chunks_per_warp) {
+                                                          T* __restrict__ y, long long z, long long chunks_per_warp,
+                                                          CooFix fx) {
   // PDL: the predecessor (zero kernel / ELL part of HYB) released us at its start; everything up to
   // the first write (or ACCUM read) of y overlaps it.
   bool waited = false;
@@ -871,11 +942,17 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long cb = warp * chunks_per_warp;
   const long long ce = cb + chunks_per_warp < nchunks ? cb + chunks_per_warp : nchunks;
+  acc_t first_piece = 0;  // FIX: this warp's piece of range_first (when it ends inside the range)
   if (cb < ce) {
     const int last_row = __ldg(row + z - 1);
     const int range_first = __ldg(row + cb * kChunk);
     int carry_row = -1;
     acc_t carry = 0;
+    // FIX: a piece of range_first is recorded, never stored (lane-uniform after the shuffles below)
+    auto emit = [&](int rr, acc_t v, bool first) {
+      if (FIX && first) first_piece += v;
+      else coo_emit<T, ACCUM>(y, rr, v, first);
+    };
     for (long long ch = cb; ch < ce; ch++) {
       const long long k = ch * kChunk + l * kCooV;
       int r[kCooV];
@@ -910,7 +987,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       // the previous chunk's carry ends exactly at this chunk boundary: emit it
       const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
       if (carry_row >= 0 && carry_row != chunk_first) {
-        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, carry_row == range_first);
+        if (l == 0) emit(carry_row, carry, carry_row == range_first);
         carry_row = -1;
         carry = 0;
       }
@@ -922,7 +999,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       for (int i = 1; i < kCooV; i++) {
         if (r[i] != cr) {
           if (in_head) { head = cur; in_head = false; }
-          else coo_emit<T, ACCUM>(y, cr, cur, cr == range_first);
+          else emit(cr, cur, cr == range_first);
           cr = r[i];
           cur = p[i];
         } else {
@@ -949,15 +1026,31 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
       if (!single) {
         const acc_t h = head + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0)));
-        coo_emit<T, ACCUM>(y, rf, h, rf == range_first);
+        emit(rf, h, rf == range_first);
       }
-      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, rl == range_first);
+      if (l < 31 && next_rf != rl) emit(rl, S, rl == range_first);
       carry_row = __shfl_sync(0xffffffffu, rl, 31);  // the chunk's last row stays open
       carry = __shfl_sync(0xffffffffu, S, 31);
     }
-    if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
+    if (FIX) {
+      // the range's first row: at most one lane emitted a piece of it per chunk; sum over the warp
+      first_piece = warp_sum(first_piece);
+      if (l == 0) {
+        fx.rrow[2 * warp] = range_first;
+        fx.rval[2 * warp] = first_piece;
+        fx.rrow[2 * warp + 1] = carry_row;
+        fx.rval[2 * warp + 1] = carry;
+        __threadfence();
+      }
+    } else if (l == 0 && carry_row >= 0) {
+      atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
+    }
+  } else if (FIX && l == 0 && warp < (long long)gridDim.x * (blockDim.x >> 5)) {
+    fx.rrow[2 * warp] = fx.rrow[2 * warp + 1] = -1;  // a warp past the last chunk: no records
+    __threadfence();
   }
   if (!waited) pdl_wait();
+  if (FIX) fix_finish<T, ACCUM>(y, fx, 2 * (long long)gridDim.x * (blockDim.x >> 5));
   pdl_trigger();
 }
 
@@ -1318,6 +1411,7 @@ struct TileWork {
   int* srow;     // row split at the start of each warp range (m: none)
   unsigned* bm;  // variants 4, 5: row-start bitmap, nchunks * 8 words
   int* ne;       // variant 5: row of each non-empty-row rank (m entries reserved)
+  CooFix fix;    // variant 4: boundary records of the one-launch kernel
 };
 TileWork tile_work(void* base, const TileGeom& g) {
   TileWork w;
@@ -1328,19 +1422,52 @@ TileWork tile_work(void* base, const TileGeom& g) {
   p += al256(sizeof(int) * g.nwarps);
   w.bm = (unsigned*)p;
   p += al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32));
-  w.ne = (int*)p;
+  w.ne = (int*)p;  // variant 5 only (m entries); variant 4 keeps its records here instead
+  const long long nrec = 2 * (g.nwarps + 8);
+  w.fix.rval = (acc_t*)p;
+  p += al256(sizeof(acc_t) * nrec);
+  w.fix.rrow = (int*)p;
+  p += al256(sizeof(int) * nrec);
+  w.fix.ticket = (unsigned*)p;
   return w;
 }
 
 // COO launch geometry: contiguous chunk ranges, one resident wave of warps at most.
-template <typename T, bool ACCUM>
-cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
+struct CooGeom {
+  long long cpw, warps, blocks;
+};
+CooGeom coo_geom(long long z) {
   const long long nchunks = ceil_div(z, kChunk);
   const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);  // <= 64 regs: 4 CTAs / SM
-  const long long cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
-  const long long warps = ceil_div(nchunks, cpw);
-  const unsigned blocks = (unsigned)ceil_div(warps, kCooThreads / 32);
-  return launch_k(k_spmv_coo<T, ACCUM>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
+  CooGeom g;
+  g.cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
+  g.warps = ceil_div(nchunks, g.cpw);
+  g.blocks = ceil_div(g.warps, kCooThreads / 32);
+  return g;
+}
+CooFix coo_fix(void* work, long long z) {
+  const CooGeom g = coo_geom(z);
+  const long long nrec = 2 * g.blocks * (kCooThreads / 32);
+  char* p = (char*)work;
+  CooFix f;
+  f.rval = (acc_t*)p;
+  p += al256(sizeof(acc_t) * nrec);
+  f.rrow = (int*)p;
+  p += al256(sizeof(int) * nrec);
+  f.ticket = (unsigned*)p;
+  return f;
+}
+
+// fix != nullptr: the one-launch kernel (no zero pass; every row holds an entry)
+template <typename T, bool ACCUM>
+cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s,
+                       void* fix = nullptr) {
+  const CooGeom g = coo_geom(z);
+  if (fix)
+    return launch_k(k_spmv_coo<T, ACCUM, true>, dim3((unsigned)g.blocks), dim3(kCooThreads), s, row, col, val, x, y,
+                    z, g.cpw, coo_fix(fix, z));
+  return launch_k(k_spmv_coo<T, ACCUM, false>, dim3((unsigned)g.blocks), dim3(kCooThreads), s, row, col, val, x, y, z,
+                  g.cpw, CooFix{nullptr, nullptr, nullptr});
 }
 
 template <typename T>
@@ -1467,20 +1594,26 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         }();
         const long long foot = 4 * (m + 1) + (4 + (long long)sizeof(T)) * z + (long long)sizeof(T) * (A->n + m);
         const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
-        auto go = [&](auto kern) {
+        const CooFix nofix{nullptr, nullptr, nullptr};
+        auto go = [&](auto kern, const CooFix& fx) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
-                          (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne);
+                          (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne, fx);
         };
         if (A->variant == 5) {  // empty rows: all of y zeroed ahead (PDL-overlapped), ranks mapped to rows
           e = launch_zero<T>(y, m, s);
           if (e == cudaSuccess)
-            e = vec ? go(k_spmv_csr_tile<T, true, true, true>) : go(k_spmv_csr_tile<T, false, true, true>);
+            e = vec ? go(k_spmv_csr_tile<T, true, true, true>, nofix) : go(k_spmv_csr_tile<T, false, true, true>, nofix);
+          break;
+        }
+        if (A->variant == 4 && A->one_launch) {  // one launch: split rows from the boundary records
+          e = vec ? go(k_spmv_csr_tile<T, true, true, false, true>, w.fix)
+                  : go(k_spmv_csr_tile<T, false, true, false, true>, w.fix);
           break;
         }
         e = launch_k(k_zero_rows<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, y, (const int*)w.srow, g.nwarps, m);
         if (e == cudaSuccess) {
-          if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>) : go(k_spmv_csr_tile<T, false, true>);
-          else e = vec ? go(k_spmv_csr_tile<T, true, false>) : go(k_spmv_csr_tile<T, false, false>);
+          if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>, nofix) : go(k_spmv_csr_tile<T, false, true>, nofix);
+          else e = vec ? go(k_spmv_csr_tile<T, true, false>, nofix) : go(k_spmv_csr_tile<T, false, false>, nofix);
         }
       } else if (A->variant == 2) {
         const long long groups = ceil_div(m, 32);
@@ -1514,6 +1647,10 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       break;
     }
     case SFS_COO: {
+      if (A->one_launch && z > 0) {  // every row holds an entry: one launch, boundary rows by the last CTA
+        e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s, A->work);
+        break;
+      }
       e = launch_zero<T>(y, m, s);
       if (e == cudaSuccess && z > 0)
         e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s);
@@ -1555,6 +1692,12 @@ __global__ void k_fill(T* __restrict__ p, long long n, T v) {
 
 }  // namespace
 
+size_t coo_fix_work_bytes(long long z) {
+  const CooGeom g = coo_geom(z);
+  const long long nrec = 2 * g.blocks * (kCooThreads / 32);
+  return al256(sizeof(acc_t) * nrec) + al256(sizeof(int) * nrec) + 256;
+}
+
 int csr_vector_tpv(long long m, long long z) {
   const long long avg = z / m;
   return avg <= 2 ? 2 : avg <= 4 ? 4 : avg <= 8 ? 8 : avg <= 16 ? 16 : 32;
@@ -1578,9 +1721,11 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 // + rank -> row map)
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
   const TileGeom g = tile_geom(z);
+  const long long nrec = 2 * (g.nwarps + 8);
   return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) +
          (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0) +
-         (bitmap == 2 ? al256(sizeof(int) * m) : 0);
+         (bitmap == 2 ? al256(sizeof(int) * m) : 0) +
+         (bitmap == 1 ? al256(sizeof(acc_t) * nrec) + al256(sizeof(int) * nrec) + 256 : 0);
 }
 
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
@@ -1609,6 +1754,11 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
     }
     k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
     count_launch();
+    if (bitmap == 1) {  // ticket of the one-launch kernel
+      e = cudaMemsetAsync(w.fix.ticket, 0, sizeof(unsigned), s);
+      count_launch();
+      if (e != cudaSuccess) return e;
+    }
     if (bitmap == 2) {
       const long long items = std::max(g.nchunks + 1, g.nwarps);
       k_tile_rank<<<grid_cap(items, 256, 8), 256, 0, s>>>(pos, m, w.a, g.nchunks, w.srow, g.nwarps);
@@ -1640,8 +1790,10 @@ int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) 
 
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
-    case SFS_CSR: return (A->variant == 1 || ((A->variant >= 3 && A->variant <= 5) && A->nnz > 0)) ? 2 : 1;
-    case SFS_COO: return A->nnz > 0 ? 2 : 1;
+    case SFS_CSR:
+      if (A->variant == 4 && A->one_launch) return 1;
+      return (A->variant == 1 || ((A->variant >= 3 && A->variant <= 5) && A->nnz > 0)) ? 2 : 1;
+    case SFS_COO: return (A->nnz > 0 && !A->one_launch) ? 2 : 1;
     case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? 2 : 1;
     default: return 1;
   }

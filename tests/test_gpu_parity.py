@@ -257,7 +257,15 @@ def test_launch_count_increases():
     c0 = sfs.launch_count()
     for _ in range(3):
         sfs.spmv(sfs.COO, M, x, y)
-    assert sfs.launch_count() - c0 == 6  # zero kernel + COO kernel per COO SpMV
+    assert sfs.launch_count() - c0 == 3  # no empty row: the one-launch COO kernel (boundary records)
+    B = cases()["rand_ragged"]  # empty rows: zero kernel + COO kernel per SpMV
+    M = sfs.convert(to_dev(B), sfs.COO)
+    x = torch.ones(B.n, dtype=torch.float64, device="cuda")
+    y = torch.empty(B.m, dtype=torch.float64, device="cuda")
+    c0 = sfs.launch_count()
+    for _ in range(3):
+        sfs.spmv(sfs.COO, M, x, y)
+    assert sfs.launch_count() - c0 == 6
 
 
 def _tile_edge_csr(dtype, cap=None, no_empty=False):
@@ -369,7 +377,10 @@ def test_csr_bitmap_tile(dtype, cap):
     x = sfsgen.vector(6, A.n, A.dtype)
     M = sfs.convert(to_dev(A), sfs.CSR, sfs.default_opts(csr_variant=4))
     assert M.layout().variant == 4
-    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="bitmap-tile")
+    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="bitmap-tile")  # one launch: split rows from the records
+    M.free()
+    M = sfs.convert(to_dev(A), sfs.COO)  # no empty row: the one-launch COO kernel
+    check_spmv(A, sfs.COO, M, x, A.dtype, ctx="coo-one-launch")
     M.free()
     B = _tile_edge_csr(dtype, cap)
     for v in (4, 5):
@@ -398,3 +409,42 @@ def test_q11_admissibility_boundary_gpu(name):
             with pytest.raises(sfs.SfsError) as ei:
                 sfs.convert(to_dev(A), fmt, opts)
             assert ei.value.status == sfs.ERR_INADMISSIBLE
+
+
+@pytest.mark.parametrize("shape", ["one_row", "two_rows", "first_last", "all_short"])
+def test_one_launch_split_rows_no_empty(shape):
+    """The one-launch COO and CSR tile (variant 4) kernels, whose rows split across warp ranges are finished
+    by the last CTA from per-warp boundary records: one row holding almost every entry (its pieces in
+    ~every warp's records), two long rows meeting mid-range, long first and last rows, and only short
+    rows (every boundary splits a row).  Every row holds >= 1 entry (the kernels' precondition)."""
+    rng = np.random.default_rng(6)
+    m, n = 40_000, 3_000_000
+    lens = np.ones(m, np.int64)
+    if shape == "one_row":
+        lens[m // 2] = 2_000_000
+    elif shape == "two_rows":
+        lens[7] = 1_234_567
+        lens[8] = 1_000_003
+    elif shape == "first_last":
+        lens[0] = 700_001
+        lens[-1] = 900_000
+    else:
+        lens[:] = rng.integers(1, 40, m)
+    rp = np.zeros(m + 1, np.int64)
+    np.cumsum(lens, out=rp[1:])
+    z = int(rp[-1])
+    col = np.empty(z, np.int64)
+    for r in range(m):
+        L = int(lens[r])
+        col[rp[r]:rp[r + 1]] = np.sort(rng.choice(n, L, replace=False)) if L > 1 else [(r * 7919) % n]
+    val = rng.uniform(0.5, 1.0, z) * rng.choice([-1.0, 1.0], z)
+    for dt in (np.float64, np.float32):
+        A = sfsgen.CSR(m, n, rp.astype(np.int32), col.astype(np.int32), val.astype(dt))
+        x = sfsgen.vector(3, n, A.dtype)
+        dA = to_dev(A)
+        for fmt, opts in [(sfs.CSR, sfs.default_opts(csr_variant=4)), (sfs.COO, None)]:
+            M = sfs.convert(dA, fmt, opts)
+            if fmt == sfs.CSR:
+                assert M.layout().variant == 4
+            check_spmv(A, fmt, M, x, A.dtype, ctx=f"{shape}/{sfs.FORMAT_NAMES[fmt]}/{np.dtype(dt).name}")
+            M.free()
