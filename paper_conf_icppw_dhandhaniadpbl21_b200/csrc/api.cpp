@@ -416,7 +416,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         const size_t wb = coo_fix_work_bytes(z);
         A->work = own(wb);
         if (!A->work) return bail(SFS_ERR_OOM, "coo records");
-        BAIL_CUDA(cudaMemsetAsync(A->work, 0, wb, s));  // ticket = 0
+        BAIL_CUDA(launch_coo_fix_prepare(r, m, z, A->work, s));
         A->one_launch = true;
       }
       break;

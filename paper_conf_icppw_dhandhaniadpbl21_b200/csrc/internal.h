@@ -104,8 +104,9 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap);
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s);
 int csr_vector_tpv(long long m, long long z);
-// one-launch COO (every row non-empty): boundary records + ticket; the ticket must start at 0
+// one-launch COO (every row non-empty): split rows at warp boundaries + their slots
 size_t coo_fix_work_bytes(long long z);
+cudaError_t launch_coo_fix_prepare(const int* row, long long m, long long z, void* work, cudaStream_t s);
 int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
 // dst[i] = src[idx[i]], i < n (exchange.cu: halo send buffers of the row-partitioned SpMV)

@@ -553,47 +553,84 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
   pdl_trigger();
 }
 
-// Boundary records of the one-launch COO and CSR tile kernels (FIX): instead of atomically adding into
-// a y zeroed by a preceding kernel (the zero / zero-rows launch), warp w writes the piece of the row
-// split at its range start (F record) and its final carry (L record); rows inside a range are stored by
-// their warp.  The last CTA to finish (acq_rel ticket) sums the records of equal rows -- the sequence
-// F0 L0 F1 L1 ... is ordered by row -- stores them and resets the ticket for the next launch.  Valid
-// only when every row holds an entry (rows the kernel never sees would stay unwritten), which the
-// handle checks at conversion.
+constexpr int kCooThreads = 256;
+constexpr int kCooV = 8;                // items per lane per step (two 128-bit loads per array)
+constexpr int kChunk = 32 * kCooV;      // items per warp step
+
+// One-launch COO and CSR tile kernels (FIX): a row split across warp ranges is finished by the warp
+// that contributes its last piece, without a zero kernel before the grid.  At handle creation every
+// split is given a slot (srow[b] = the row holding the first entry of warp b's range when it started
+// before it; a run of boundaries b1..b2 splitting one row shares slot b1 and expects b2 - b1 + 2
+// pieces: warp b1 - 1's final carry, whole ranges b1..b2 - 1, warp b2's first piece).  A contributing
+// warp adds its piece into the slot's fp64 accumulator, fences, and counts itself in; the warp that
+// completes the count takes the sum (and zeroes the slot for the next launch) and stores y[row].  Rows
+// inside a range are stored directly.  Valid only when every row holds an entry (rows the kernel never
+// sees would stay unwritten): the handle checks nnz_min >= 1.
 struct CooFix {
-  int* rrow;        // 2 * nwarps
-  acc_t* rval;      // 2 * nwarps
-  unsigned* ticket; // 1
+  const int* srow;      // nwarps: split row at each warp's range start (m: none)
+  const int* slot;      // nwarps: slot of boundary b (run start), -1: none
+  const int* expected;  // nwarps: pieces expected at a run-start slot
+  acc_t* acc;           // nwarps
+  unsigned* cnt;        // nwarps
 };
 
-template <typename T, bool ACCUM>
-__device__ void coo_fixup(T* __restrict__ y, const CooFix& fx, long long nrec) {
-  for (long long i = threadIdx.x; i < nrec; i += blockDim.x) {
-    const int r = __ldcg(fx.rrow + i);
-    if (r < 0 || (i > 0 && __ldcg(fx.rrow + i - 1) == r)) continue;  // not the first record of its row
-    acc_t v = 0;
-    for (long long j = i; j < nrec && __ldcg(fx.rrow + j) == r; j++) v += __ldcg(fx.rval + j);
-    if (ACCUM) y[r] = (T)((acc_t)y[r] + v);
-    else y[r] = (T)v;
+template <typename T>
+__device__ __forceinline__ void fix_contribute(T* __restrict__ y, const CooFix& fx, int slot, int row, acc_t v) {
+  atomicAdd(fx.acc + slot, v);
+  __threadfence();
+  const unsigned c = atomicAdd(fx.cnt + slot, 1u);
+  if ((int)c + 1 == __ldg(fx.expected + slot)) {  // the last piece: every other add is visible
+    __threadfence();
+    const acc_t t = __longlong_as_double(atomicExch((unsigned long long*)(fx.acc + slot), 0ull));
+    fx.cnt[slot] = 0u;
+    y[row] = (T)t;
   }
 }
 
-// Every thread of the grid calls this after its records are written (and fenced): the last CTA applies
-// them.
-template <typename T, bool ACCUM>
-__device__ __forceinline__ void fix_finish(T* __restrict__ y, const CooFix& fx, long long nrec) {
-  __shared__ bool s_last;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    unsigned prev;
-    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev) : "l"(fx.ticket) : "memory");
-    s_last = prev == gridDim.x - 1;
+// A warp's boundary pieces (lane 0): `first` = its pieces of the row split at its range start (valid when
+// srow[warp] < m), `last` = its final carry of row `last_row` when that row continues into warp + 1.
+template <typename T>
+__device__ __forceinline__ void fix_warp_end(T* __restrict__ y, const CooFix& fx, long long warp, long long nwarps,
+                                             long long m, acc_t first, int last_row, acc_t last, bool cont) {
+  const int sf = __ldg(fx.srow + warp) < (int)m ? __ldg(fx.slot + warp) : -1;
+  const int sl = cont && warp + 1 < nwarps ? __ldg(fx.slot + warp + 1) : -1;
+  if (sf >= 0 && sf == sl) {  // the range lies inside one split row: one piece
+    fix_contribute<T>(y, fx, sf, last_row, first + last);
+    return;
   }
-  __syncthreads();
-  if (s_last) {
-    __threadfence();
-    coo_fixup<T, ACCUM>(y, fx, nrec);
-    if (threadIdx.x == 0) *fx.ticket = 0u;
+  if (sf >= 0) fix_contribute<T>(y, fx, sf, __ldg(fx.srow + warp), first);
+  if (sl >= 0) fix_contribute<T>(y, fx, sl, last_row, last);
+}
+
+// slots of the split rows (handle creation): one thread per boundary b >= 1
+__global__ void k_fix_slots(const int* __restrict__ srow, long long nwarps, long long m, int* __restrict__ slot,
+                            int* __restrict__ expected, acc_t* __restrict__ acc, unsigned* __restrict__ cnt) {
+  for (long long b = (long long)blockIdx.x * blockDim.x + threadIdx.x; b < nwarps; b += (long long)gridDim.x * blockDim.x) {
+    acc[b] = 0;
+    cnt[b] = 0;
+    expected[b] = 0;
+    const int r = b > 0 ? srow[b] : (int)m;
+    if (r >= (int)m) {
+      slot[b] = -1;
+      continue;
+    }
+    long long b1 = b;
+    while (b1 - 1 >= 1 && srow[b1 - 1] == r) b1--;
+    slot[b] = (int)b1;
+    if (b1 == b) {
+      long long b2 = b;
+      while (b2 + 1 < nwarps && srow[b2 + 1] == r) b2++;
+      expected[b] = (int)(b2 - b1 + 2);
+    }
+  }
+}
+
+// COO: srow[w] = the row of warp w's first entry if the entry before it has the same row, else m
+__global__ void k_coo_split_rows(const int* __restrict__ row, long long z, long long cpw, long long nwarps, long long m,
+                                 int* __restrict__ srow) {
+  for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nwarps; w += (long long)gridDim.x * blockDim.x) {
+    const long long k = w * cpw * kChunk;
+    srow[w] = (w > 0 && k < z && row[k - 1] == row[k]) ? row[k] : (int)m;
   }
 }
 
@@ -820,18 +857,11 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     open = __shfl_sync(0xffffffffu, S, 31);
   }
   if constexpr (FIX) {
-    static_assert(!MAP, "records hold row ids");
+    static_assert(!MAP, "slots hold row ids");
     const bool cont = open_row >= 0 && open_row == next_split;  // continues past the range (lane-uniform)
     if (l == 0 && open_row >= 0 && !cont) emit(open_row, open_row, open);
     split_piece = warp_sum(split_piece);
-    if (l == 0) {
-      const int sr = __ldg(srow + warp);  // the row split at this range's start (m: none)
-      fx.rrow[2 * warp] = sr < (int)m ? sr : -1;
-      fx.rval[2 * warp] = split_piece;
-      fx.rrow[2 * warp + 1] = cont ? open_row : -1;
-      fx.rval[2 * warp + 1] = cont ? open : acc_t(0);
-      __threadfence();
-    }
+    if (l == 0) fix_warp_end<T>(y, fx, warp, nwarps, m, split_piece, open_row, open, cont);
     return;
   }
   if (l == 0 && open_row >= 0) {  // a piece of a split row if it continues past the range
@@ -857,12 +887,7 @@ __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __res
                                         s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne, fx);
   } else {
     pdl_wait();
-    if (FIX && (threadIdx.x & 31) == 0) {  // a warp past the last range: no records
-      fx.rrow[2 * warp] = fx.rrow[2 * warp + 1] = -1;
-      __threadfence();
-    }
   }
-  if (FIX) fix_finish<T, false>(y, fx, 2 * (long long)gridDim.x * (blockDim.x >> 5));
   pdl_trigger();
 }
 
@@ -918,9 +943,6 @@ __global__ void k_tile_rank(const int* __restrict__ pos, long long m, int* __res
 }
 
 // ======================================================================== COO (also the COO part of HYB)
-constexpr int kCooThreads = 256;
-constexpr int kCooV = 8;                // items per lane per step (two 128-bit loads per array)
-constexpr int kChunk = 32 * kCooV;      // items per warp step
 
 template <typename T, bool ACCUM>
 __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
@@ -930,10 +952,10 @@ __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
 }
 
 template <typename T, bool ACCUM, bool FIX = false>
-__global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
+__global__ void __launch_bounds__(kCooThreads, 4) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
                                                           T* __restrict__ y, long long z, long long chunks_per_warp,
-                                                          CooFix fx) {
+                                                          CooFix fx, long long m_rows) {
   // PDL: the predecessor (zero kernel / ELL part of HYB) released us at its start; everything up to
   // the first write (or ACCUM read) of y overlaps it.
   bool waited = false;
@@ -942,16 +964,24 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long cb = warp * chunks_per_warp;
   const long long ce = cb + chunks_per_warp < nchunks ? cb + chunks_per_warp : nchunks;
-  acc_t first_piece = 0;  // FIX: this warp's piece of range_first (when it ends inside the range)
+  acc_t first_piece = 0;  // FIX: this warp's pieces of range_first when that row is split
+  const long long nwarps_fix = ceil_div(nchunks, chunks_per_warp);
+  const long long m_fix = m_rows;
   if (cb < ce) {
     const int last_row = __ldg(row + z - 1);
     const int range_first = __ldg(row + cb * kChunk);
+    // FIX: range_first is split iff it started in the previous range (slot-finished); otherwise every
+    // row of this range is complete or continues out of it, and complete rows are stored plainly
+    const bool split_first = FIX && __ldg(fx.srow + warp) < (int)m_rows;
     int carry_row = -1;
     acc_t carry = 0;
-    // FIX: a piece of range_first is recorded, never stored (lane-uniform after the shuffles below)
     auto emit = [&](int rr, acc_t v, bool first) {
-      if (FIX && first) first_piece += v;
-      else coo_emit<T, ACCUM>(y, rr, v, first);
+      if (FIX) {
+        if (first && split_first) first_piece += v;
+        else coo_emit<T, ACCUM>(y, rr, v, false);
+      } else {
+        coo_emit<T, ACCUM>(y, rr, v, first);
+      }
     };
     for (long long ch = cb; ch < ce; ch++) {
       const long long k = ch * kChunk + l * kCooV;
@@ -1033,24 +1063,22 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       carry = __shfl_sync(0xffffffffu, S, 31);
     }
     if (FIX) {
-      // the range's first row: at most one lane emitted a piece of it per chunk; sum over the warp
+      // pieces of a split range_first row (recorded, lane-local) summed over the warp; the final carry is
+      // stored when its row ends with the range, else it is the warp's last piece of a split row
       first_piece = warp_sum(first_piece);
+      const bool cont = carry_row >= 0 && warp + 1 < nwarps_fix && __ldg(fx.srow + warp + 1) == carry_row;
       if (l == 0) {
-        fx.rrow[2 * warp] = range_first;
-        fx.rval[2 * warp] = first_piece;
-        fx.rrow[2 * warp + 1] = carry_row;
-        fx.rval[2 * warp + 1] = carry;
-        __threadfence();
+        if (carry_row >= 0 && !cont) {
+          if (carry_row == range_first && split_first) first_piece += carry;
+          else coo_emit<T, ACCUM>(y, carry_row, carry, false);
+        }
+        fix_warp_end<T>(y, fx, warp, nwarps_fix, m_fix, first_piece, carry_row, carry, cont);
       }
     } else if (l == 0 && carry_row >= 0) {
       atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
     }
-  } else if (FIX && l == 0 && warp < (long long)gridDim.x * (blockDim.x >> 5)) {
-    fx.rrow[2 * warp] = fx.rrow[2 * warp + 1] = -1;  // a warp past the last chunk: no records
-    __threadfence();
   }
   if (!waited) pdl_wait();
-  if (FIX) fix_finish<T, ACCUM>(y, fx, 2 * (long long)gridDim.x * (blockDim.x >> 5));
   pdl_trigger();
 }
 
@@ -1413,6 +1441,26 @@ struct TileWork {
   int* ne;       // variant 5: row of each non-empty-row rank (m entries reserved)
   CooFix fix;    // variant 4: boundary records of the one-launch kernel
 };
+// slot arrays of the one-launch kernels at p (nw warps): slot, expected, acc, cnt
+CooFix fix_layout(char* p, long long nw, const int* srow) {
+  CooFix f;
+  f.srow = srow;
+  f.acc = (acc_t*)p;
+  p += al256(sizeof(acc_t) * nw);
+  f.slot = (const int*)p;
+  p += al256(sizeof(int) * nw);
+  f.expected = (const int*)p;
+  p += al256(sizeof(int) * nw);
+  f.cnt = (unsigned*)p;
+  return f;
+}
+size_t fix_bytes(long long nw) { return al256(sizeof(acc_t) * nw) + 3 * al256(sizeof(int) * nw); }
+cudaError_t launch_fix_slots(const CooFix& f, long long nw, long long m, cudaStream_t s) {
+  k_fix_slots<<<grid_cap(nw, 256, 8), 256, 0, s>>>(f.srow, nw, m, (int*)f.slot, (int*)f.expected, f.acc, f.cnt);
+  count_launch();
+  return cudaGetLastError();
+}
+
 TileWork tile_work(void* base, const TileGeom& g) {
   TileWork w;
   char* p = (char*)base;
@@ -1422,13 +1470,8 @@ TileWork tile_work(void* base, const TileGeom& g) {
   p += al256(sizeof(int) * g.nwarps);
   w.bm = (unsigned*)p;
   p += al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32));
-  w.ne = (int*)p;  // variant 5 only (m entries); variant 4 keeps its records here instead
-  const long long nrec = 2 * (g.nwarps + 8);
-  w.fix.rval = (acc_t*)p;
-  p += al256(sizeof(acc_t) * nrec);
-  w.fix.rrow = (int*)p;
-  p += al256(sizeof(int) * nrec);
-  w.fix.ticket = (unsigned*)p;
+  w.ne = (int*)p;  // variant 5 only (m entries); variant 4 keeps its split-row slots here instead
+  w.fix = fix_layout(p, g.nwarps, w.srow);
   return w;
 }
 
@@ -1445,29 +1488,22 @@ CooGeom coo_geom(long long z) {
   g.blocks = ceil_div(g.warps, kCooThreads / 32);
   return g;
 }
+// COO one-launch work: srow[nwarps] then the slot arrays
 CooFix coo_fix(void* work, long long z) {
   const CooGeom g = coo_geom(z);
-  const long long nrec = 2 * g.blocks * (kCooThreads / 32);
-  char* p = (char*)work;
-  CooFix f;
-  f.rval = (acc_t*)p;
-  p += al256(sizeof(acc_t) * nrec);
-  f.rrow = (int*)p;
-  p += al256(sizeof(int) * nrec);
-  f.ticket = (unsigned*)p;
-  return f;
+  return fix_layout((char*)work + al256(sizeof(int) * g.warps), g.warps, (const int*)work);
 }
 
 // fix != nullptr: the one-launch kernel (no zero pass; every row holds an entry)
 template <typename T, bool ACCUM>
 cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s,
-                       void* fix = nullptr) {
+                       void* fix = nullptr, long long m = 0) {
   const CooGeom g = coo_geom(z);
   if (fix)
     return launch_k(k_spmv_coo<T, ACCUM, true>, dim3((unsigned)g.blocks), dim3(kCooThreads), s, row, col, val, x, y,
-                    z, g.cpw, coo_fix(fix, z));
+                    z, g.cpw, coo_fix(fix, z), m);
   return launch_k(k_spmv_coo<T, ACCUM, false>, dim3((unsigned)g.blocks), dim3(kCooThreads), s, row, col, val, x, y, z,
-                  g.cpw, CooFix{nullptr, nullptr, nullptr});
+                  g.cpw, CooFix{nullptr, nullptr, nullptr, nullptr, nullptr}, m);
 }
 
 template <typename T>
@@ -1594,7 +1630,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         }();
         const long long foot = 4 * (m + 1) + (4 + (long long)sizeof(T)) * z + (long long)sizeof(T) * (A->n + m);
         const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
-        const CooFix nofix{nullptr, nullptr, nullptr};
+        const CooFix nofix{nullptr, nullptr, nullptr, nullptr, nullptr};
         auto go = [&](auto kern, const CooFix& fx) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
                           (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne, fx);
@@ -1648,7 +1684,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
     }
     case SFS_COO: {
       if (A->one_launch && z > 0) {  // every row holds an entry: one launch, boundary rows by the last CTA
-        e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s, A->work);
+        e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s, A->work, m);
         break;
       }
       e = launch_zero<T>(y, m, s);
@@ -1694,8 +1730,15 @@ __global__ void k_fill(T* __restrict__ p, long long n, T v) {
 
 size_t coo_fix_work_bytes(long long z) {
   const CooGeom g = coo_geom(z);
-  const long long nrec = 2 * g.blocks * (kCooThreads / 32);
-  return al256(sizeof(acc_t) * nrec) + al256(sizeof(int) * nrec) + 256;
+  return al256(sizeof(int) * g.warps) + fix_bytes(g.warps);
+}
+
+cudaError_t launch_coo_fix_prepare(const int* row, long long m, long long z, void* work, cudaStream_t s) {
+  const CooGeom g = coo_geom(z);
+  k_coo_split_rows<<<grid_cap(g.warps, 256, 8), 256, 0, s>>>(row, z, g.cpw, g.warps, m, (int*)work);
+  count_launch();
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? launch_fix_slots(coo_fix(work, z), g.warps, m, s) : e;
 }
 
 int csr_vector_tpv(long long m, long long z) {
@@ -1721,11 +1764,9 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 // + rank -> row map)
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
   const TileGeom g = tile_geom(z);
-  const long long nrec = 2 * (g.nwarps + 8);
   return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) +
          (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0) +
-         (bitmap == 2 ? al256(sizeof(int) * m) : 0) +
-         (bitmap == 1 ? al256(sizeof(acc_t) * nrec) + al256(sizeof(int) * nrec) + 256 : 0);
+         (bitmap == 2 ? al256(sizeof(int) * m) : 0) + (bitmap == 1 ? fix_bytes(g.nwarps) : 0);
 }
 
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
@@ -1754,9 +1795,8 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
     }
     k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
     count_launch();
-    if (bitmap == 1) {  // ticket of the one-launch kernel
-      e = cudaMemsetAsync(w.fix.ticket, 0, sizeof(unsigned), s);
-      count_launch();
+    if (bitmap == 1) {  // split-row slots of the one-launch kernel
+      e = launch_fix_slots(w.fix, g.nwarps, m, s);
       if (e != cudaSuccess) return e;
     }
     if (bitmap == 2) {
