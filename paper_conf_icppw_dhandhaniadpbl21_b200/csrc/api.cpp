@@ -330,15 +330,6 @@ static sfs_status features_finish(const DevCSR& d, const sfs_race_opts& o, const
   return SFS_OK;
 }
 
-// SFS_ONE_LAUNCH=0: keep the zero-kernel pairs of COO and the CSR tile kernel (A/B switch)
-static bool one_launch_enabled() {
-  static const bool v = [] {
-    const char* e = getenv("SFS_ONE_LAUNCH");
-    return !(e && e[0] == '0');
-  }();
-  return v;
-}
-
 // ---------------------------------------------------------------- conversion
 static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_features_t& f, const FeatWork& fw,
                                Matrix** out, cudaStream_t s) {
@@ -401,7 +392,6 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
         A->work = own(csr_tile_work_bytes(m, z, bitmap));
         if (!A->work) return bail(SFS_ERR_OOM, "csr tile partition");
         BAIL_CUDA(launch_csr_tile_prepare((const int*)A->ptr[0], m, z, A->work, bitmap, s));
-        A->one_launch = A->variant == 4 && one_launch_enabled();
       }
       break;
     }
@@ -412,13 +402,6 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       if (!r || !c || !v) return bail(SFS_ERR_OOM, "coo");
       BAIL_CUDA(launch_csr2coo(d.dtype, d.rp, d.col, d.val, m, z, r, c, v, s));
       A->ptr[0] = r; A->ptr[1] = c; A->ptr[2] = v;
-      if (z > 0 && f.nnz_min >= 1 && one_launch_enabled()) {  // no empty row: one launch (boundary records)
-        const size_t wb = coo_fix_work_bytes(z);
-        A->work = own(wb);
-        if (!A->work) return bail(SFS_ERR_OOM, "coo records");
-        BAIL_CUDA(launch_coo_fix_prepare(r, m, z, A->work, s));
-        A->one_launch = true;
-      }
       break;
     }
     case SFS_ELL: {

@@ -553,87 +553,6 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
   pdl_trigger();
 }
 
-constexpr int kCooThreads = 256;
-constexpr int kCooV = 8;                // items per lane per step (two 128-bit loads per array)
-constexpr int kChunk = 32 * kCooV;      // items per warp step
-
-// One-launch COO and CSR tile kernels (FIX): a row split across warp ranges is finished by the warp
-// that contributes its last piece, without a zero kernel before the grid.  At handle creation every
-// split is given a slot (srow[b] = the row holding the first entry of warp b's range when it started
-// before it; a run of boundaries b1..b2 splitting one row shares slot b1 and expects b2 - b1 + 2
-// pieces: warp b1 - 1's final carry, whole ranges b1..b2 - 1, warp b2's first piece).  A contributing
-// warp adds its piece into the slot's fp64 accumulator, fences, and counts itself in; the warp that
-// completes the count takes the sum (and zeroes the slot for the next launch) and stores y[row].  Rows
-// inside a range are stored directly.  Valid only when every row holds an entry (rows the kernel never
-// sees would stay unwritten): the handle checks nnz_min >= 1.
-struct CooFix {
-  const int* srow;      // nwarps: split row at each warp's range start (m: none)
-  const int* slot;      // nwarps: slot of boundary b (run start), -1: none
-  const int* expected;  // nwarps: pieces expected at a run-start slot
-  acc_t* acc;           // nwarps
-  unsigned* cnt;        // nwarps
-};
-
-template <typename T>
-__device__ __forceinline__ void fix_contribute(T* __restrict__ y, const CooFix& fx, int slot, int row, acc_t v) {
-  atomicAdd(fx.acc + slot, v);
-  __threadfence();
-  const unsigned c = atomicAdd(fx.cnt + slot, 1u);
-  if ((int)c + 1 == __ldg(fx.expected + slot)) {  // the last piece: every other add is visible
-    __threadfence();
-    const acc_t t = __longlong_as_double(atomicExch((unsigned long long*)(fx.acc + slot), 0ull));
-    fx.cnt[slot] = 0u;
-    y[row] = (T)t;
-  }
-}
-
-// A warp's boundary pieces (lane 0): `first` = its pieces of the row split at its range start (valid when
-// srow[warp] < m), `last` = its final carry of row `last_row` when that row continues into warp + 1.
-template <typename T>
-__device__ __forceinline__ void fix_warp_end(T* __restrict__ y, const CooFix& fx, long long warp, long long nwarps,
-                                             long long m, acc_t first, int last_row, acc_t last, bool cont) {
-  const int sf = __ldg(fx.srow + warp) < (int)m ? __ldg(fx.slot + warp) : -1;
-  const int sl = cont && warp + 1 < nwarps ? __ldg(fx.slot + warp + 1) : -1;
-  if (sf >= 0 && sf == sl) {  // the range lies inside one split row: one piece
-    fix_contribute<T>(y, fx, sf, last_row, first + last);
-    return;
-  }
-  if (sf >= 0) fix_contribute<T>(y, fx, sf, __ldg(fx.srow + warp), first);
-  if (sl >= 0) fix_contribute<T>(y, fx, sl, last_row, last);
-}
-
-// slots of the split rows (handle creation): one thread per boundary b >= 1
-__global__ void k_fix_slots(const int* __restrict__ srow, long long nwarps, long long m, int* __restrict__ slot,
-                            int* __restrict__ expected, acc_t* __restrict__ acc, unsigned* __restrict__ cnt) {
-  for (long long b = (long long)blockIdx.x * blockDim.x + threadIdx.x; b < nwarps; b += (long long)gridDim.x * blockDim.x) {
-    acc[b] = 0;
-    cnt[b] = 0;
-    expected[b] = 0;
-    const int r = b > 0 ? srow[b] : (int)m;
-    if (r >= (int)m) {
-      slot[b] = -1;
-      continue;
-    }
-    long long b1 = b;
-    while (b1 - 1 >= 1 && srow[b1 - 1] == r) b1--;
-    slot[b] = (int)b1;
-    if (b1 == b) {
-      long long b2 = b;
-      while (b2 + 1 < nwarps && srow[b2 + 1] == r) b2++;
-      expected[b] = (int)(b2 - b1 + 2);
-    }
-  }
-}
-
-// COO: srow[w] = the row of warp w's first entry if the entry before it has the same row, else m
-__global__ void k_coo_split_rows(const int* __restrict__ row, long long z, long long cpw, long long nwarps, long long m,
-                                 int* __restrict__ srow) {
-  for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nwarps; w += (long long)gridDim.x * blockDim.x) {
-    const long long k = w * cpw * kChunk;
-    srow[w] = (w > 0 && k < z && row[k - 1] == row[k]) ? row[k] : (int)m;
-  }
-}
-
 // ======================================================================== CSR tile (nnz-balanced)
 // The COO kernel's shape on the CSR arrays.  Warp w streams the contiguous chunks [cb, ce) of 256
 // entries (8 per lane, 256-bit col/val loads whose addresses do not depend on row_ptr), and the row of
@@ -692,13 +611,13 @@ __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, lo
 // ne[j] maps rank j to its row; y was zeroed whole ahead of this grid (the empty rows stay 0), so no
 // per-chunk row_ptr walk is needed (variant 3's walk over runs of empty rows made it 3x slower than the
 // merge path on R-MAT).
-template <typename T, bool VEC, bool BM = false, bool MAP = false, bool FIX = false>
+template <typename T, bool VEC, bool BM = false, bool MAP = false>
 __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const int* __restrict__ col,
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
                                               const int* __restrict__ ca, const int* __restrict__ srow,
                                               long long nwarps, int* head, const unsigned* __restrict__ bm, int pf,
-                                              const int* __restrict__ ne, const CooFix& fx) {
+                                              const int* __restrict__ ne) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
   const long long cb = warp * cpw;
@@ -713,14 +632,9 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
   bool waited = false;                // PDL: loads of the first chunk overlap k_zero_rows
   // emit(row, y index, value); MAP: the y index of a lane's first / last row is loaded as soon as the
   // ranks are known (off the store path), rows strictly inside a lane's 8 entries (rare) load it there
-  acc_t split_piece = 0;  // FIX: this lane's pieces of the row split at the range start (< own_lo)
   auto emit = [&](int row, int yr, acc_t v) {
-    if (row < own_lo) {  // the piece of the row carried into this range
-      if (FIX) split_piece += v;
-      else atomicAdd(y + yr, (T)v);
-    } else {
-      y[yr] = (T)v;
-    }
+    if (row < own_lo) atomicAdd(y + yr, (T)v);  // the piece of the row carried into this range
+    else y[yr] = (T)v;
   };
   int a_run = own_lo;  // BM: first row starting at or after the chunk start
   for (long long ch = cb; ch < ce; ch++) {
@@ -856,14 +770,6 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     if (MAP) open_y = __shfl_sync(0xffffffffu, yl, 31);
     open = __shfl_sync(0xffffffffu, S, 31);
   }
-  if constexpr (FIX) {
-    static_assert(!MAP, "slots hold row ids");
-    const bool cont = open_row >= 0 && open_row == next_split;  // continues past the range (lane-uniform)
-    if (l == 0 && open_row >= 0 && !cont) emit(open_row, open_row, open);
-    split_piece = warp_sum(split_piece);
-    if (l == 0) fix_warp_end<T>(y, fx, warp, nwarps, m, split_piece, open_row, open, cont);
-    return;
-  }
   if (l == 0 && open_row >= 0) {  // a piece of a split row if it continues past the range
     const int oy = MAP ? open_y : open_row;
     if (open_row == next_split) atomicAdd(y + oy, (T)open);
@@ -872,22 +778,21 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
 }
 
 // blockDim is 64, 128 or 256 (smaller CTAs spread a small matrix's few warps over more SMs)
-template <typename T, bool VEC, bool BM, bool MAP = false, bool FIX = false>
+template <typename T, bool VEC, bool BM, bool MAP = false>
 __global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
                                                                const int* __restrict__ ca, const int* __restrict__ srow,
                                                                const unsigned* __restrict__ bm, int pf,
-                                                               const int* __restrict__ ne, CooFix fx) {
+                                                               const int* __restrict__ ne) {
   __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  if (warp < nwarps) {
-    csr_tile_warp<T, VEC, BM, MAP, FIX>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps,
-                                        s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne, fx);
-  } else {
+  if (warp < nwarps)
+    csr_tile_warp<T, VEC, BM, MAP>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps,
+                                   s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne);
+  else
     pdl_wait();
-  }
   pdl_trigger();
 }
 
@@ -943,6 +848,9 @@ __global__ void k_tile_rank(const int* __restrict__ pos, long long m, int* __res
 }
 
 // ======================================================================== COO (also the COO part of HYB)
+constexpr int kCooThreads = 256;
+constexpr int kCooV = 8;                // items per lane per step (two 128-bit loads per array)
+constexpr int kChunk = 32 * kCooV;      // items per warp step
 
 template <typename T, bool ACCUM>
 __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
@@ -951,11 +859,10 @@ __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
   else y[row] = (T)v;
 }
 
-template <typename T, bool ACCUM, bool FIX = false>
-__global__ void __launch_bounds__(kCooThreads, 4) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
+template <typename T, bool ACCUM>
+__global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
-                                                          T* __restrict__ y, long long z, long long chunks_per_warp,
-                                                          CooFix fx, long long m_rows) {
+                                                          T* __restrict__ y, long long z, long long chunks_per_warp) {
   // PDL: the predecessor (zero kernel / ELL part of HYB) released us at its start; everything up to
   // the first write (or ACCUM read) of y overlaps it.
   bool waited = false;
@@ -964,25 +871,11 @@ __global__ void __launch_bounds__(kCooThreads, 4) k_spmv_coo(const int* __restri
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const long long cb = warp * chunks_per_warp;
   const long long ce = cb + chunks_per_warp < nchunks ? cb + chunks_per_warp : nchunks;
-  acc_t first_piece = 0;  // FIX: this warp's pieces of range_first when that row is split
-  const long long nwarps_fix = ceil_div(nchunks, chunks_per_warp);
-  const long long m_fix = m_rows;
   if (cb < ce) {
     const int last_row = __ldg(row + z - 1);
     const int range_first = __ldg(row + cb * kChunk);
-    // FIX: range_first is split iff it started in the previous range (slot-finished); otherwise every
-    // row of this range is complete or continues out of it, and complete rows are stored plainly
-    const bool split_first = FIX && __ldg(fx.srow + warp) < (int)m_rows;
     int carry_row = -1;
     acc_t carry = 0;
-    auto emit = [&](int rr, acc_t v, bool first) {
-      if (FIX) {
-        if (first && split_first) first_piece += v;
-        else coo_emit<T, ACCUM>(y, rr, v, false);
-      } else {
-        coo_emit<T, ACCUM>(y, rr, v, first);
-      }
-    };
     for (long long ch = cb; ch < ce; ch++) {
       const long long k = ch * kChunk + l * kCooV;
       int r[kCooV];
@@ -1017,7 +910,7 @@ __global__ void __launch_bounds__(kCooThreads, 4) k_spmv_coo(const int* __restri
       // the previous chunk's carry ends exactly at this chunk boundary: emit it
       const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
       if (carry_row >= 0 && carry_row != chunk_first) {
-        if (l == 0) emit(carry_row, carry, carry_row == range_first);
+        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, carry_row == range_first);
         carry_row = -1;
         carry = 0;
       }
@@ -1029,7 +922,7 @@ __global__ void __launch_bounds__(kCooThreads, 4) k_spmv_coo(const int* __restri
       for (int i = 1; i < kCooV; i++) {
         if (r[i] != cr) {
           if (in_head) { head = cur; in_head = false; }
-          else emit(cr, cur, cr == range_first);
+          else coo_emit<T, ACCUM>(y, cr, cur, cr == range_first);
           cr = r[i];
           cur = p[i];
         } else {
@@ -1056,27 +949,13 @@ __global__ void __launch_bounds__(kCooThreads, 4) k_spmv_coo(const int* __restri
       const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
       if (!single) {
         const acc_t h = head + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0)));
-        emit(rf, h, rf == range_first);
+        coo_emit<T, ACCUM>(y, rf, h, rf == range_first);
       }
-      if (l < 31 && next_rf != rl) emit(rl, S, rl == range_first);
+      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, rl == range_first);
       carry_row = __shfl_sync(0xffffffffu, rl, 31);  // the chunk's last row stays open
       carry = __shfl_sync(0xffffffffu, S, 31);
     }
-    if (FIX) {
-      // pieces of a split range_first row (recorded, lane-local) summed over the warp; the final carry is
-      // stored when its row ends with the range, else it is the warp's last piece of a split row
-      first_piece = warp_sum(first_piece);
-      const bool cont = carry_row >= 0 && warp + 1 < nwarps_fix && __ldg(fx.srow + warp + 1) == carry_row;
-      if (l == 0) {
-        if (carry_row >= 0 && !cont) {
-          if (carry_row == range_first && split_first) first_piece += carry;
-          else coo_emit<T, ACCUM>(y, carry_row, carry, false);
-        }
-        fix_warp_end<T>(y, fx, warp, nwarps_fix, m_fix, first_piece, carry_row, carry, cont);
-      }
-    } else if (l == 0 && carry_row >= 0) {
-      atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
-    }
+    if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
   }
   if (!waited) pdl_wait();
   pdl_trigger();
@@ -1439,28 +1318,7 @@ struct TileWork {
   int* srow;     // row split at the start of each warp range (m: none)
   unsigned* bm;  // variants 4, 5: row-start bitmap, nchunks * 8 words
   int* ne;       // variant 5: row of each non-empty-row rank (m entries reserved)
-  CooFix fix;    // variant 4: boundary records of the one-launch kernel
 };
-// slot arrays of the one-launch kernels at p (nw warps): slot, expected, acc, cnt
-CooFix fix_layout(char* p, long long nw, const int* srow) {
-  CooFix f;
-  f.srow = srow;
-  f.acc = (acc_t*)p;
-  p += al256(sizeof(acc_t) * nw);
-  f.slot = (const int*)p;
-  p += al256(sizeof(int) * nw);
-  f.expected = (const int*)p;
-  p += al256(sizeof(int) * nw);
-  f.cnt = (unsigned*)p;
-  return f;
-}
-size_t fix_bytes(long long nw) { return al256(sizeof(acc_t) * nw) + 3 * al256(sizeof(int) * nw); }
-cudaError_t launch_fix_slots(const CooFix& f, long long nw, long long m, cudaStream_t s) {
-  k_fix_slots<<<grid_cap(nw, 256, 8), 256, 0, s>>>(f.srow, nw, m, (int*)f.slot, (int*)f.expected, f.acc, f.cnt);
-  count_launch();
-  return cudaGetLastError();
-}
-
 TileWork tile_work(void* base, const TileGeom& g) {
   TileWork w;
   char* p = (char*)base;
@@ -1470,40 +1328,19 @@ TileWork tile_work(void* base, const TileGeom& g) {
   p += al256(sizeof(int) * g.nwarps);
   w.bm = (unsigned*)p;
   p += al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32));
-  w.ne = (int*)p;  // variant 5 only (m entries); variant 4 keeps its split-row slots here instead
-  w.fix = fix_layout(p, g.nwarps, w.srow);
+  w.ne = (int*)p;
   return w;
 }
 
 // COO launch geometry: contiguous chunk ranges, one resident wave of warps at most.
-struct CooGeom {
-  long long cpw, warps, blocks;
-};
-CooGeom coo_geom(long long z) {
+template <typename T, bool ACCUM>
+cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
   const long long nchunks = ceil_div(z, kChunk);
   const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);  // <= 64 regs: 4 CTAs / SM
-  CooGeom g;
-  g.cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
-  g.warps = ceil_div(nchunks, g.cpw);
-  g.blocks = ceil_div(g.warps, kCooThreads / 32);
-  return g;
-}
-// COO one-launch work: srow[nwarps] then the slot arrays
-CooFix coo_fix(void* work, long long z) {
-  const CooGeom g = coo_geom(z);
-  return fix_layout((char*)work + al256(sizeof(int) * g.warps), g.warps, (const int*)work);
-}
-
-// fix != nullptr: the one-launch kernel (no zero pass; every row holds an entry)
-template <typename T, bool ACCUM>
-cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s,
-                       void* fix = nullptr, long long m = 0) {
-  const CooGeom g = coo_geom(z);
-  if (fix)
-    return launch_k(k_spmv_coo<T, ACCUM, true>, dim3((unsigned)g.blocks), dim3(kCooThreads), s, row, col, val, x, y,
-                    z, g.cpw, coo_fix(fix, z), m);
-  return launch_k(k_spmv_coo<T, ACCUM, false>, dim3((unsigned)g.blocks), dim3(kCooThreads), s, row, col, val, x, y, z,
-                  g.cpw, CooFix{nullptr, nullptr, nullptr, nullptr, nullptr}, m);
+  const long long cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
+  const long long warps = ceil_div(nchunks, cpw);
+  const unsigned blocks = (unsigned)ceil_div(warps, kCooThreads / 32);
+  return launch_k(k_spmv_coo<T, ACCUM>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
 }
 
 template <typename T>
@@ -1630,26 +1467,20 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         }();
         const long long foot = 4 * (m + 1) + (4 + (long long)sizeof(T)) * z + (long long)sizeof(T) * (A->n + m);
         const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
-        const CooFix nofix{nullptr, nullptr, nullptr, nullptr, nullptr};
-        auto go = [&](auto kern, const CooFix& fx) {
+        auto go = [&](auto kern) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
-                          (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne, fx);
+                          (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne);
         };
         if (A->variant == 5) {  // empty rows: all of y zeroed ahead (PDL-overlapped), ranks mapped to rows
           e = launch_zero<T>(y, m, s);
           if (e == cudaSuccess)
-            e = vec ? go(k_spmv_csr_tile<T, true, true, true>, nofix) : go(k_spmv_csr_tile<T, false, true, true>, nofix);
-          break;
-        }
-        if (A->variant == 4 && A->one_launch) {  // one launch: split rows from the boundary records
-          e = vec ? go(k_spmv_csr_tile<T, true, true, false, true>, w.fix)
-                  : go(k_spmv_csr_tile<T, false, true, false, true>, w.fix);
+            e = vec ? go(k_spmv_csr_tile<T, true, true, true>) : go(k_spmv_csr_tile<T, false, true, true>);
           break;
         }
         e = launch_k(k_zero_rows<T>, dim3(grid_cap(g.nwarps, 256, 4)), dim3(256), s, y, (const int*)w.srow, g.nwarps, m);
         if (e == cudaSuccess) {
-          if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>, nofix) : go(k_spmv_csr_tile<T, false, true>, nofix);
-          else e = vec ? go(k_spmv_csr_tile<T, true, false>, nofix) : go(k_spmv_csr_tile<T, false, false>, nofix);
+          if (A->variant == 4) e = vec ? go(k_spmv_csr_tile<T, true, true>) : go(k_spmv_csr_tile<T, false, true>);
+          else e = vec ? go(k_spmv_csr_tile<T, true, false>) : go(k_spmv_csr_tile<T, false, false>);
         }
       } else if (A->variant == 2) {
         const long long groups = ceil_div(m, 32);
@@ -1683,10 +1514,6 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       break;
     }
     case SFS_COO: {
-      if (A->one_launch && z > 0) {  // every row holds an entry: one launch, boundary rows by the last CTA
-        e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s, A->work, m);
-        break;
-      }
       e = launch_zero<T>(y, m, s);
       if (e == cudaSuccess && z > 0)
         e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s);
@@ -1728,19 +1555,6 @@ __global__ void k_fill(T* __restrict__ p, long long n, T v) {
 
 }  // namespace
 
-size_t coo_fix_work_bytes(long long z) {
-  const CooGeom g = coo_geom(z);
-  return al256(sizeof(int) * g.warps) + fix_bytes(g.warps);
-}
-
-cudaError_t launch_coo_fix_prepare(const int* row, long long m, long long z, void* work, cudaStream_t s) {
-  const CooGeom g = coo_geom(z);
-  k_coo_split_rows<<<grid_cap(g.warps, 256, 8), 256, 0, s>>>(row, z, g.cpw, g.warps, m, (int*)work);
-  count_launch();
-  cudaError_t e = cudaGetLastError();
-  return e == cudaSuccess ? launch_fix_slots(coo_fix(work, z), g.warps, m, s) : e;
-}
-
 int csr_vector_tpv(long long m, long long z) {
   const long long avg = z / m;
   return avg <= 2 ? 2 : avg <= 4 ? 4 : avg <= 8 ? 8 : avg <= 16 ? 16 : 32;
@@ -1766,7 +1580,7 @@ size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
   const TileGeom g = tile_geom(z);
   return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) +
          (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0) +
-         (bitmap == 2 ? al256(sizeof(int) * m) : 0) + (bitmap == 1 ? fix_bytes(g.nwarps) : 0);
+         (bitmap == 2 ? al256(sizeof(int) * m) : 0);
 }
 
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
@@ -1795,10 +1609,6 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
     }
     k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
     count_launch();
-    if (bitmap == 1) {  // split-row slots of the one-launch kernel
-      e = launch_fix_slots(w.fix, g.nwarps, m, s);
-      if (e != cudaSuccess) return e;
-    }
     if (bitmap == 2) {
       const long long items = std::max(g.nchunks + 1, g.nwarps);
       k_tile_rank<<<grid_cap(items, 256, 8), 256, 0, s>>>(pos, m, w.a, g.nchunks, w.srow, g.nwarps);
@@ -1830,10 +1640,8 @@ int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z) 
 
 int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
-    case SFS_CSR:
-      if (A->variant == 4 && A->one_launch) return 1;
-      return (A->variant == 1 || ((A->variant >= 3 && A->variant <= 5) && A->nnz > 0)) ? 2 : 1;
-    case SFS_COO: return (A->nnz > 0 && !A->one_launch) ? 2 : 1;
+    case SFS_CSR: return (A->variant == 1 || ((A->variant >= 3 && A->variant <= 5) && A->nnz > 0)) ? 2 : 1;
+    case SFS_COO: return A->nnz > 0 ? 2 : 1;
     case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? 2 : 1;
     default: return 1;
   }

@@ -257,15 +257,7 @@ def test_launch_count_increases():
     c0 = sfs.launch_count()
     for _ in range(3):
         sfs.spmv(sfs.COO, M, x, y)
-    assert sfs.launch_count() - c0 == 3  # no empty row: the one-launch COO kernel (boundary records)
-    B = cases()["rand_ragged"]  # empty rows: zero kernel + COO kernel per SpMV
-    M = sfs.convert(to_dev(B), sfs.COO)
-    x = torch.ones(B.n, dtype=torch.float64, device="cuda")
-    y = torch.empty(B.m, dtype=torch.float64, device="cuda")
-    c0 = sfs.launch_count()
-    for _ in range(3):
-        sfs.spmv(sfs.COO, M, x, y)
-    assert sfs.launch_count() - c0 == 6
+    assert sfs.launch_count() - c0 == 6  # zero kernel + COO kernel per COO SpMV
 
 
 def _tile_edge_csr(dtype, cap=None, no_empty=False):
@@ -377,10 +369,10 @@ def test_csr_bitmap_tile(dtype, cap):
     x = sfsgen.vector(6, A.n, A.dtype)
     M = sfs.convert(to_dev(A), sfs.CSR, sfs.default_opts(csr_variant=4))
     assert M.layout().variant == 4
-    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="bitmap-tile")  # one launch: split rows from the records
+    check_spmv(A, sfs.CSR, M, x, A.dtype, ctx="bitmap-tile")
     M.free()
-    M = sfs.convert(to_dev(A), sfs.COO)  # no empty row: the one-launch COO kernel
-    check_spmv(A, sfs.COO, M, x, A.dtype, ctx="coo-one-launch")
+    M = sfs.convert(to_dev(A), sfs.COO)
+    check_spmv(A, sfs.COO, M, x, A.dtype, ctx="coo-no-empty-rows")
     M.free()
     B = _tile_edge_csr(dtype, cap)
     for v in (4, 5):
@@ -412,11 +404,10 @@ def test_q11_admissibility_boundary_gpu(name):
 
 
 @pytest.mark.parametrize("shape", ["one_row", "two_rows", "first_last", "all_short"])
-def test_one_launch_split_rows_no_empty(shape):
-    """The one-launch COO and CSR tile (variant 4) kernels, whose rows split across warp ranges are finished
-    by the last CTA from per-warp boundary records: one row holding almost every entry (its pieces in
-    ~every warp's records), two long rows meeting mid-range, long first and last rows, and only short
-    rows (every boundary splits a row).  Every row holds >= 1 entry (the kernels' precondition)."""
+def test_split_rows_no_empty(shape):
+    """COO and the bitmap CSR tile kernel (variant 4, which needs every row non-empty) on rows split across
+    warp ranges: one row holding almost every entry (pieces in ~every warp range), two long rows meeting
+    mid-range, long first and last rows, and only short rows (every boundary splits a row)."""
     rng = np.random.default_rng(6)
     m, n = 40_000, 3_000_000
     lens = np.ones(m, np.int64)
