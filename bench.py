@@ -442,6 +442,9 @@ def run_ours(args):
         if gloo:
             dist.init_process_group("gloo")
         else:
+            # communicator set-up logged (NVLS / P2P transports), not per-call traffic
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     dev = torch.device("cuda", local)
     cdev = torch.device("cpu") if gloo else dev  # where the collectives' tensors live

@@ -118,7 +118,7 @@ def lib():
                    "sfs_matrix_describe"):
             getattr(L, fn).restype = _I32
         _lib = L
-        if os.environ.get("SFS_TORCH_ALLOC", "1") != "0":
+        if os.environ.get("SFS_TORCH_ALLOC", "0") == "1":
             use_torch_allocator(True)
     return _lib
 
@@ -135,7 +135,10 @@ EXPORTED = ["sfs_features", "sfs_convert", "sfs_spmv", "sfs_label_corpus", "sfs_
 # on ANOTHER stream (host inputs are staged on the copy stream and released on the compute stream) is
 # handed back only once an event recorded on the freeing stream has completed (the deferred-free
 # discipline of torch's record_stream; nothing waits, so the copy / race overlap is kept).
-# SFS_TORCH_ALLOC=0 keeps the library's own CUDA stream-ordered pool.
+# Opt-in (use_torch_allocator() or SFS_TORCH_ALLOC=1): every library allocation becomes a Python call
+# under the GIL, which the device-resident race hides (bench 162.9 vs 162.7 matrices/s) but the
+# chunk-synchronised host-input path does not (e2e 127 vs 161 matrices/s, profiles/r02/micro_ab.txt);
+# by default the library keeps its own CUDA stream-ordered pool.
 _ALLOC_T = ctypes.CFUNCTYPE(_P, ctypes.c_size_t, _P)
 _FREE_T = ctypes.CFUNCTYPE(None, _P, _P)
 _alloc_state = {"on": False, "blocks": {}, "pending": [], "cbs": None}

@@ -2,9 +2,10 @@
 //
 // SpMV is HBM-bound (0.10–0.46 flop/B): every kernel streams the format's arrays once with
 // L1-bypassing loads (ld.global.nc.L1::no_allocate) and gathers x through L1/L2 (__ldg).  No tensor
-// cores: the path is not a dense contraction.  Products and sums are formed in fp64 for both value
-// types (an fp32 product is exact in fp64), so fp32 rows of ~10^5 entries stay within the 1e-5
-// per-row tolerance; y is rounded once to its dtype.
+// cores: the path is not a dense contraction.  Sums run in fp64 for both value types; fp64 values form
+// fp64 products, fp32 values form each product (or a chain of <= 8 products of one row) in fp32 and
+// widen it once (mulp below), so fp32 rows of any length stay far inside the 1e-5 per-row tolerance;
+// y is rounded once to its dtype.
 //
 // Two regimes shape every launch: matrices far larger than the GPU's in-flight capacity are
 // bandwidth-bound (one wave, each thread streaming a long slice); L2-resident / mid-size matrices
@@ -39,6 +40,23 @@ namespace sfs {
 namespace {
 
 typedef double acc_t;
+
+// Products.  fp64 values: fp64 products.  fp32 values: the product is formed in fp32 (one rounding,
+// relative error <= 2^-24) and widened once, and the sums run in fp64 -- per row the error stays below
+// (2^-24 + K 2^-53) |A||x|, far inside the 1e-5 fp32 tolerance for any row length K, at one conversion
+// per entry instead of two.  The row-owning fp32 kernels (DIA, ELL) go further: a batch of <= 8
+// entries of a row is chained in fp32 FMAs and widened once (error <= 8 * 2^-24 |A||x| per batch).
+// -DSFS_FP64_PRODUCTS restores fp64 products everywhere (A/B).
+#ifdef SFS_FP64_PRODUCTS
+constexpr bool kFp32Arith = false;
+#else
+constexpr bool kFp32Arith = true;
+#endif
+__device__ __forceinline__ acc_t mulp(double a, double b) { return a * b; }
+__device__ __forceinline__ acc_t mulp(float a, float b) {
+  if constexpr (kFp32Arith) return (acc_t)__fmul_rn(a, b);
+  return (acc_t)a * (acc_t)b;
+}
 
 constexpr long long kResidentThreads = (long long)kSMs * 2048;
 
@@ -249,10 +267,10 @@ __device__ __forceinline__ acc_t csr_row_partial(const int* __restrict__ col, co
   for (; k + TPV < e; k += 2 * TPV) {
     const int c0 = ld_stream(col + k), c1 = ld_stream(col + k + TPV);
     const T v0 = ld_stream(val + k), v1 = ld_stream(val + k + TPV);
-    s += (acc_t)v0 * (acc_t)ld_x(x + c0);
-    s += (acc_t)v1 * (acc_t)ld_x(x + c1);
+    s += mulp(v0, ld_x(x + c0));
+    s += mulp(v1, ld_x(x + c1));
   }
-  if (k < e) s += (acc_t)ld_stream(val + k) * (acc_t)ld_x(x + ld_stream(col + k));
+  if (k < e) s += mulp(ld_stream(val + k), ld_x(x + ld_stream(col + k)));
   return s;
 }
 
@@ -357,7 +375,7 @@ __global__ void __launch_bounds__(kSThreads, stream_ctas<T>()) k_spmv_csr_stream
 #pragma unroll
       for (int u = 0; u < kSU; u++) {
         const int i = u * 32 + lane;
-        if (i < n) buf[i] = (acc_t)v[u] * (acc_t)xv[u];
+        if (i < n) buf[i] = mulp(v[u], xv[u]);
       }
       __syncwarp();
       const int lo = (b > w0 ? b : w0) - w0, hi = (e < w0 + n ? e : w0 + n) - w0;
@@ -500,7 +518,7 @@ __global__ void __launch_bounds__(kMT) k_spmv_csr_merge(const int* __restrict__ 
 #pragma unroll
     for (int u = 0; u < kMI; u++) {
       const int i = threadIdx.x + u * kMT;
-      if (i < nk) s_prod[i] = (acc_t)vv[u] * (acc_t)xv[u];
+      if (i < nk) s_prod[i] = mulp(vv[u], xv[u]);
     }
   }
   __syncthreads();
@@ -670,7 +688,7 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
         }
       }
 #pragma unroll
-      for (int i = 0; i < kTV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
+      for (int i = 0; i < kTV; i++) p[i] = mulp(v[i], ld_x(x + c[i]));
     }
     if (!waited) {
       pdl_wait();
@@ -888,13 +906,13 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
         ld_stream8(col + k, c);
         ld_stream8(val + k, v);
 #pragma unroll
-        for (int i = 0; i < kCooV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
+        for (int i = 0; i < kCooV; i++) p[i] = mulp(v[i], ld_x(x + c[i]));
       } else {
 #pragma unroll
         for (int i = 0; i < kCooV; i++) {
           if (k + i < z) {
             r[i] = ld_stream(row + k + i);
-            p[i] = (acc_t)ld_stream(val + k + i) * (acc_t)ld_x(x + ld_stream(col + k + i));
+            p[i] = mulp(ld_stream(val + k + i), ld_x(x + ld_stream(col + k + i)));
           } else {
             r[i] = last_row;  // padding joins the last segment with value 0
             p[i] = 0;
@@ -1019,22 +1037,35 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
           c[u] = ld_stream4(cp + (long long)(j + u) * P);
           v[u].load_stream(vp + (long long)(j + u) * P);
         }
+        if constexpr (sizeof(T) == 4 && kFp32Arith) {  // the batch's products per row chained in fp32
+          float t[4] = {0.f, 0.f, 0.f, 0.f};
 #pragma unroll
-        for (int u = 0; u < kB; u++) {
-          if (c[u].x >= 0) acc[0] += (acc_t)v[u].v[0] * (acc_t)ld_x(x + c[u].x);
-          if (c[u].y >= 0) acc[1] += (acc_t)v[u].v[1] * (acc_t)ld_x(x + c[u].y);
-          if (c[u].z >= 0) acc[2] += (acc_t)v[u].v[2] * (acc_t)ld_x(x + c[u].z);
-          if (c[u].w >= 0) acc[3] += (acc_t)v[u].v[3] * (acc_t)ld_x(x + c[u].w);
+          for (int u = 0; u < kB; u++) {
+            if (c[u].x >= 0) t[0] = __fmaf_rn(v[u].v[0], ld_x(x + c[u].x), t[0]);
+            if (c[u].y >= 0) t[1] = __fmaf_rn(v[u].v[1], ld_x(x + c[u].y), t[1]);
+            if (c[u].z >= 0) t[2] = __fmaf_rn(v[u].v[2], ld_x(x + c[u].z), t[2]);
+            if (c[u].w >= 0) t[3] = __fmaf_rn(v[u].v[3], ld_x(x + c[u].w), t[3]);
+          }
+#pragma unroll
+          for (int q = 0; q < 4; q++) acc[q] += (acc_t)t[q];
+        } else {
+#pragma unroll
+          for (int u = 0; u < kB; u++) {
+            if (c[u].x >= 0) acc[0] += mulp(v[u].v[0], ld_x(x + c[u].x));
+            if (c[u].y >= 0) acc[1] += mulp(v[u].v[1], ld_x(x + c[u].y));
+            if (c[u].z >= 0) acc[2] += mulp(v[u].v[2], ld_x(x + c[u].z));
+            if (c[u].w >= 0) acc[3] += mulp(v[u].v[3], ld_x(x + c[u].w));
+          }
         }
       }
       for (; j < j1; j++) {
         const int4 c = ld_stream4(cp + (long long)j * P);
         Vec4<T> v;
         v.load_stream(vp + (long long)j * P);
-        if (c.x >= 0) acc[0] += (acc_t)v.v[0] * (acc_t)ld_x(x + c.x);
-        if (c.y >= 0) acc[1] += (acc_t)v.v[1] * (acc_t)ld_x(x + c.y);
-        if (c.z >= 0) acc[2] += (acc_t)v.v[2] * (acc_t)ld_x(x + c.z);
-        if (c.w >= 0) acc[3] += (acc_t)v.v[3] * (acc_t)ld_x(x + c.w);
+        if (c.x >= 0) acc[0] += mulp(v.v[0], ld_x(x + c.x));
+        if (c.y >= 0) acc[1] += mulp(v.v[1], ld_x(x + c.y));
+        if (c.z >= 0) acc[2] += mulp(v.v[2], ld_x(x + c.z));
+        if (c.w >= 0) acc[3] += mulp(v.v[3], ld_x(x + c.w));
       }
       if (OVF) {
         // the 4 rows' overflow entries are contiguous: [ob[0], ob[4]); batches of 4 (clamped loads),
@@ -1057,7 +1088,7 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
           }
 #pragma unroll
           for (int u = 0; u < 4; u++) {
-            const acc_t t = (acc_t)v[u] * (acc_t)ld_x(x + c[u]);
+            const acc_t t = mulp(v[u], ld_x(x + c[u]));
             const int kk = k + u;
             if (kk < ob[4]) {
               if (kk < ob[1]) acc[0] += t;
@@ -1161,7 +1192,7 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 #pragma unroll
         for (int u = 0; u < kB; u++)
 #pragma unroll
-          for (int q = 0; q < kR; q++) acc[q] += (acc_t)v[u][q] * (acc_t)xv[u][q];
+          for (int q = 0; q < kR; q++) acc[q] += mulp(v[u][q], xv[u][q]);
       } else {
         for (int u = 0; u < nb; u++) {
           const T* vp = dval + (long long)(d + u) * P + r0;
@@ -1169,7 +1200,7 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 #pragma unroll
           for (int q = 0; q < kR; q++) {
             const long long rr = r0 + q * G, c = c0 + q * G;
-            if (rr < m && c >= 0 && c < n) acc[q] += (acc_t)ld_stream(vp + q * G) * (acc_t)ld_x(x + c);
+            if (rr < m && c >= 0 && c < n) acc[q] += mulp(ld_stream(vp + q * G), ld_x(x + c));
           }
         }
       }
@@ -1257,10 +1288,20 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
 #pragma unroll
             for (int q = 0; q < 4; q++) xv[u][q] = ld_x(xp + q);
           }
+          if constexpr (sizeof(T) == 4 && kFp32Arith) {  // the batch's products per row chained in fp32
 #pragma unroll
-          for (int u = 0; u < kB; u++)
+            for (int q = 0; q < 4; q++) {
+              float t = __fmul_rn(v[0].v[q], xv[0][q]);
 #pragma unroll
-            for (int q = 0; q < 4; q++) acc[q] += (acc_t)v[u].v[q] * (acc_t)xv[u][q];
+              for (int u = 1; u < kB; u++) t = __fmaf_rn(v[u].v[q], xv[u][q], t);
+              acc[q] += (acc_t)t;
+            }
+          } else {
+#pragma unroll
+            for (int u = 0; u < kB; u++)
+#pragma unroll
+              for (int q = 0; q < 4; q++) acc[q] += mulp(v[u].v[q], xv[u][q]);
+          }
         } else {
           for (int u = 0; u < nb; u++) {
             Vec4<T> v;
@@ -1268,7 +1309,7 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
 #pragma unroll
             for (int q = 0; q < 4; q++) {
               const long long c = r0 + q + off[u];
-              if (r0 + q < m && c >= 0 && c < n) acc[q] += (acc_t)v.v[q] * (acc_t)ld_x(x + c);
+              if (r0 + q < m && c >= 0 && c < n) acc[q] += mulp(v.v[q], ld_x(x + c));
             }
           }
         }

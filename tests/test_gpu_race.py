@@ -86,7 +86,8 @@ def test_torch_allocator_hook_owns_library_buffers():
     A = _mats()["band"]
     x = sfsgen.vector(11, A.n)
     dA = to_dev(A)
-    assert sfs.torch_allocator_enabled()
+    was = sfs.torch_allocator_enabled()
+    sfs.use_torch_allocator(True)
     torch.cuda.synchronize()
     before = torch.cuda.memory_allocated()
     M = sfs.convert(dA, sfs.ELL)
@@ -103,7 +104,7 @@ def test_torch_allocator_hook_owns_library_buffers():
         y_pool = check_spmv(A, sfs.ELL, M2, x, sfs.F64, "library pool")
         M2.free()
     finally:
-        sfs.use_torch_allocator(True)
+        sfs.use_torch_allocator(was)
     assert np.array_equal(y_hook, y_pool)
 
 
@@ -115,8 +116,13 @@ def test_torch_allocator_host_inputs_cross_stream():
     pin = lambda a: torch.from_numpy(np.ascontiguousarray(a)).pin_memory()
     hm = [sfs.Csr(B.m, B.n, pin(B.rp), pin(B.col), pin(B.val)) for B in A.values()]
     opts = sfs.default_opts(reps=3, warmup=1)
-    f1, l1 = sfs.label_corpus(hm, opts)
-    f2, l2 = sfs.label_corpus(hm, opts)
+    was = sfs.torch_allocator_enabled()
+    sfs.use_torch_allocator(True)
+    try:
+        f1, l1 = sfs.label_corpus(hm, opts)
+        f2, l2 = sfs.label_corpus(hm, opts)
+    finally:
+        sfs.use_torch_allocator(was)
     for k, a, b, L1, L2 in zip(A, f1, f2, l1, l2):
         assert_features_equal(a, oracle.features(A[k].m, A[k].n, A[k].rp, A[k].col), k)
         assert_features_equal(b, a, k)
