@@ -687,8 +687,11 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
           v[i] = k + i < z ? ld_stream(val + kk) : T(0);
         }
       }
+      T xv[kTV];  // every gather issued before the first product (memory-level parallelism)
 #pragma unroll
-      for (int i = 0; i < kTV; i++) p[i] = mulp(v[i], ld_x(x + c[i]));
+      for (int i = 0; i < kTV; i++) xv[i] = ld_x(x + c[i]);
+#pragma unroll
+      for (int i = 0; i < kTV; i++) p[i] = mulp(v[i], xv[i]);
     }
     if (!waited) {
       pdl_wait();
@@ -905,14 +908,17 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
         ld_stream8(row + k, r);  // 32 B aligned: k is a multiple of 8 and the arrays are ours
         ld_stream8(col + k, c);
         ld_stream8(val + k, v);
+        // fp64 products here even for fp32 values: the fp32-product build of this kernel measured slower on
+        // R-MAT 2^22 (286 vs 243 us: ptxas drops to 48 registers and the chunk loop loses its overlap;
+        // profiles/r02/micro_ab.txt)
 #pragma unroll
-        for (int i = 0; i < kCooV; i++) p[i] = mulp(v[i], ld_x(x + c[i]));
+        for (int i = 0; i < kCooV; i++) p[i] = (acc_t)v[i] * (acc_t)ld_x(x + c[i]);
       } else {
 #pragma unroll
         for (int i = 0; i < kCooV; i++) {
           if (k + i < z) {
             r[i] = ld_stream(row + k + i);
-            p[i] = mulp(ld_stream(val + k + i), ld_x(x + ld_stream(col + k + i)));
+            p[i] = (acc_t)ld_stream(val + k + i) * (acc_t)ld_x(x + ld_stream(col + k + i));
           } else {
             r[i] = last_row;  // padding joins the last segment with value 0
             p[i] = 0;
