@@ -1239,12 +1239,13 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 // (the ELL mapping; warp = 128 consecutive rows, 512 contiguous bytes per slab load) and its 4 x values
 // are 4 scalar loads hitting the same lines (L1).  fp32's scalar strided mapping above moves 4 bytes
 // per load instruction; this one moves 16.  S diagonal-parts per row block meet in shared memory.
-template <typename T, int S, bool PUSH>
+template <typename T, int S, bool PUSH, bool XA = false>
 __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __restrict__ offs,
                                                                 const T* __restrict__ dval,
                                                                 const T* __restrict__ x, T* __restrict__ y,
                                                                 long long m, long long n, long long P, int nd,
                                                                 PushParam<PUSH> push, int pfd) {
+  static_assert(!XA || sizeof(T) == 4, "XA: fp32 x");
   constexpr int G = kDiaThreads / S;
   constexpr int kB = sizeof(T) == 4 ? 4 : 2;  // diagonals per batch (register cap)
   __shared__ int s_off[kDiaSmemOffs];
@@ -1291,8 +1292,26 @@ __global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __res
 #pragma unroll
           for (int u = 0; u < kB; u++) {
             const T* xp = x + r0 + off[u];
+            if constexpr (XA) {
+              // the 4 x values in the widest aligned pieces (x 16 B aligned, r0 a multiple of 4, so the
+              // alignment s = off mod 4 is warp-uniform): s = 0 one 16-byte load, s = 2 two 8-byte loads,
+              // s odd 4 + 8 + 4 bytes -- a lane-strided warp load costs ~4 L1 wavefronts whatever its width
+              const int sft = off[u] & 3;
+              if (sft == 0) {
+                const float4 a = __ldg(reinterpret_cast<const float4*>(xp));
+                xv[u][0] = a.x; xv[u][1] = a.y; xv[u][2] = a.z; xv[u][3] = a.w;
+              } else if (sft == 2) {
+                const float2 a = __ldg(reinterpret_cast<const float2*>(xp));
+                const float2 b = __ldg(reinterpret_cast<const float2*>(xp + 2));
+                xv[u][0] = a.x; xv[u][1] = a.y; xv[u][2] = b.x; xv[u][3] = b.y;
+              } else {
+                const float2 a = __ldg(reinterpret_cast<const float2*>(xp + 1));
+                xv[u][0] = ld_x(xp); xv[u][1] = a.x; xv[u][2] = a.y; xv[u][3] = ld_x(xp + 3);
+              }
+            } else {
 #pragma unroll
-            for (int q = 0; q < 4; q++) xv[u][q] = ld_x(xp + q);
+              for (int q = 0; q < 4; q++) xv[u][q] = ld_x(xp + q);
+            }
           }
           if constexpr (sizeof(T) == 4 && kFp32Arith) {  // the batch's products per row chained in fp32
 #pragma unroll
@@ -1466,6 +1485,21 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
       return e ? atoi(e) : 1;
     }();
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
+    if constexpr (sizeof(T) == 4) {
+      static const bool xa = [] {  // SFS_DIA_XA=0: 4 scalar x loads per diagonal (A/B)
+        const char* e = getenv("SFS_DIA_XA");
+        return !(e && e[0] == '0');
+      }();
+      if (xa && ((uintptr_t)x % 16) == 0) {
+        switch (S) {
+          case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          case 4: return launch_k(k_spmv_dia_v4<T, 4, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          case 8: return launch_k(k_spmv_dia_v4<T, 8, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+          default: return launch_k(k_spmv_dia_v4<T, 16, PUSH, true>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
+        }
+      }
+    }
     switch (S) {
       case 1: return launch_k(k_spmv_dia_v4<T, 1, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
       case 2: return launch_k(k_spmv_dia_v4<T, 2, PUSH>, gd, bd, s, offs, dv, x, y, m, A->n, A->pitch, nd, push, pfd);
