@@ -62,6 +62,8 @@ def parse():
     p.add_argument("--rowpart-N", type=int, default=128, help="configs[3] grid edge (0 = skip the rowpart record)")
     p.add_argument("--rowpart-iters", type=int, default=100)
     p.add_argument("--predictor-nc", type=int, default=20, help="clusters of the f2 subset-labelling record (0 = skip)")
+    p.add_argument("--no-configs-record", dest="configs_record", action="store_false",
+                   help="skip the configs[0] / configs[2] race record")
     return p.parse_args()
 
 
@@ -426,6 +428,46 @@ def rowpart_measure(N, iters, warmup, rank, world, dev, gloo, group=None, format
     return out
 
 
+# ------------------------------------------------------------------ configs[0] / configs[2] race lines
+def configs_measure(dev):
+    """BASELINE configs[0] (2D 5-point Laplacian 64x64, fp64, all formats) and configs[2] (R-MAT 2^22, fp32;
+    CSR / COO / HYB, ELL and DIA inadmissible) through sfs_label_corpus: the race protocol (5 warm-ups +
+    100 back-to-back reps between CUDA events) and, for configs[2], the cold protocol (L2 flushed
+    before every rep, SURVEY §8(d) "Roofline timing"); GB/s on the algorithmic bytes of each format.  The
+    R-MAT matrix is generated on the device (bit-identical to the host generator)."""
+    import torch
+
+    import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
+    import sfsgen
+    out = {}
+    A = sfsgen.laplace2d(64)
+    t = lambda a: torch.from_numpy(a).to(dev)
+    c0 = sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), t(sfsgen.vector(5, A.n)))
+    try:
+        m, n, rp, col, val = sfsgen.generate_device(sfsgen.make_spec(sfsgen.RMAT, seed=1, ia=22, ib=16, dtype=sfsgen.F32))
+        c2 = sfs.Csr(m, n, rp, col, val, sfsgen.vector_device(5, n, sfsgen.F32))
+        gen = "device"
+    except Exception:
+        B = sfsgen.rmat(22, seed=1)
+        c2 = sfs.Csr(B.m, B.n, t(B.rp), t(B.col), t(B.val), t(sfsgen.vector(5, B.n, sfsgen.F32)))
+        gen = "host"
+    for name, M, cold in (("configs[0] 2D 5-pt Laplacian 64x64 fp64", c0, False),
+                          ("configs[2] R-MAT 2^22 fp32", c2, True)):
+        rec = {"nrows": M.m, "nnz": M.nnz}
+        modes = [("hot", 0)] + ([("cold", 1)] if cold else [])
+        for mode, flag in modes:
+            feats, labs = sfs.label_corpus([M], sfs.default_opts(cold=flag))
+            L, F = labs[0], feats[0]
+            rec[mode] = {sfs.FORMAT_NAMES[f]: {"t_spmv_us": L["t_spmv_us"][f], "gbs": L["bytes"][f] / L["t_spmv_us"][f] / 1e3}
+                         for f in range(5) if L["status"][f] == 0}
+            rec[mode + "_label"] = sfs.FORMAT_NAMES[L["label"]] if L["label"] >= 0 else None
+        rec["admissible"] = [sfs.FORMAT_NAMES[f] for f in range(5) if (F["admissible_mask"] >> f) & 1]
+        rec["csr_variant"] = F["csr_variant"]
+        out[name] = rec
+    out["generation"] = f"configs[2] generated on the {gen}"
+    return out
+
+
 # ------------------------------------------------------------------ our arm
 def run_ours(args):
     import torch
@@ -672,6 +714,14 @@ def run_ours(args):
         except Exception as ex:  # reported in the line, never silently dropped
             rowpart = {"error": f"{type(ex).__name__}: {ex}"[:400]}
 
+    # ---- configs[0] / configs[2] race lines (rank 0, N = 1)
+    configs = None
+    if rank == 0 and world == 1 and args.configs_record:
+        try:
+            configs = configs_measure(dev)
+        except Exception as ex:
+            configs = {"error": f"{type(ex).__name__}: {ex}"[:300]}
+
     # ---- CPU oracle baseline (rank 0, N = 1 only)
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -698,7 +748,7 @@ def run_ours(args):
                 "e2e": e2e, "gpu_launches": launches_all, "clocks": clk, "roofline": roofline,
                 "cpu_baseline": cpu, "per_format": per_fmt,
                 "label_histogram": {k: v["labels"] for k, v in per_fmt.items()},
-                "predictor": predictor, "rowpart": rowpart}
+                "predictor": predictor, "rowpart": rowpart, "configs_0_2": configs}
         s = json.dumps(line)
         print(s, flush=True)
         if args.out:
