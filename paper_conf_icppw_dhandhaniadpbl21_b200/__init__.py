@@ -190,8 +190,9 @@ def use_torch_allocator(enable: bool = True):
     """Route the library's device allocations through torch's caching allocator (sfs_set_allocator)."""
     L = lib()
     if enable and not _alloc_state["on"]:
-        cbs = (_ALLOC_T(_torch_alloc), _FREE_T(_torch_free))
-        _alloc_state["cbs"] = cbs  # keep the trampolines alive while the library may call them
+        if _alloc_state["cbs"] is None:  # created once: handles built under the hook keep calling its free
+            _alloc_state["cbs"] = (_ALLOC_T(_torch_alloc), _FREE_T(_torch_free))
+        cbs = _alloc_state["cbs"]
         L.sfs_set_allocator(cbs[0], cbs[1])
         _alloc_state["on"] = True
     elif not enable and _alloc_state["on"]:

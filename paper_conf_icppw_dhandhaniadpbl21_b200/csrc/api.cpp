@@ -86,6 +86,14 @@ void dfree(void* p, cudaStream_t s) {
   cudaFreeAsync(p, s);
 }
 
+// A handle outlives the call that built it: its buffers go back to the allocator that provided them,
+// even if sfs_set_allocator changed in between.
+static void dfree_from(void* p, cudaStream_t s, void (*user_free)(void*, void*)) {
+  if (!p) return;
+  if (user_free) user_free(p, (void*)s);
+  else cudaFreeAsync(p, s);
+}
+
 // RAII list of stream-ordered temporaries
 struct Temps {
   cudaStream_t s;
@@ -342,6 +350,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
   A->pitch = pitch_of(d.m);
   A->stream = s;
   A->variant = f.csr_variant;
+  A->user_free = g_user_free;  // the allocator this handle's buffers come from
   const size_t sv = vbytes(d.dtype);
   auto own = [&](size_t b) -> void* {
     void* p = dalloc(b, s);
@@ -473,7 +482,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
 
 static void matrix_free(Matrix* A) {
   if (!A) return;
-  for (int i = 0; i < A->n_owned; i++) dfree(A->owned[i], A->stream);
+  for (int i = 0; i < A->n_owned; i++) dfree_from(A->owned[i], A->stream, A->user_free);
   delete A;
 }
 

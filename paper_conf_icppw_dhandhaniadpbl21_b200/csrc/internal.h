@@ -138,6 +138,7 @@ struct Matrix {
                                // HYB: 1 = one launch (ptr[5] = ovf)
   void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;
+  void (*user_free)(void*, void*) = nullptr;  // allocator hook at creation (nullptr: the library's pool)
 };
 
 }  // namespace sfs

@@ -106,6 +106,16 @@ def test_torch_allocator_hook_owns_library_buffers():
     finally:
         sfs.use_torch_allocator(was)
     assert np.array_equal(y_hook, y_pool)
+    # a handle keeps the allocator it was built with: built under the hook, freed after the hook is off
+    sfs.use_torch_allocator(True)
+    M3 = sfs.convert(dA, sfs.COO)
+    sfs.use_torch_allocator(False)
+    torch.cuda.synchronize()
+    held = torch.cuda.memory_allocated()
+    M3.free()
+    torch.cuda.synchronize()
+    assert torch.cuda.memory_allocated() < held  # returned to torch's pool, not to the library's
+    sfs.use_torch_allocator(was)
 
 
 def test_torch_allocator_host_inputs_cross_stream():
