@@ -34,6 +34,9 @@ sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402
 
+# ncu hot-rep traffic of the race per format (tools/traffic_corpus.py); the newest round's file
+TRAFFIC_JSON = next((p for p in (os.path.join(ROOT, "profiles", r, "traffic_corpus200.json") for r in ("r02", "r01"))
+                     if os.path.exists(p)), os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json"))
 METRIC = "matrices labelled/s (features + all-format conversion + 100-rep SpMV race + label), corpus-200"
 UNIT = "matrices/s"
 DAGGR_BYTES = 136  # device aggregate record copied back per matrix (internal.h DevAggr)
@@ -620,7 +623,7 @@ def run_ours(args):
                  if L["status"][f] == 0 and L["status"][0] == 0 and L["t_spmv_us"][0] > 0]) if f else 0.0),
         }
     try:  # per-format L2-sector rate from the ncu sector counts of the same race (profiles/r01/traffic_corpus200.json)
-        with open(os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json")) as fh:
+        with open(TRAFFIC_JSON) as fh:
             tjall = json.load(fh)
         for k, v in per_fmt.items():
             tk = tjall.get(k)
@@ -648,13 +651,13 @@ def run_ours(args):
     bytes_per_launch = (per_fmt[dom]["gbs"] * 1e9 * per_fmt[dom]["spmv_time_s"] / launches_dom) if launches_dom else 0
     traffic, traffic_src = None, None
     try:  # ncu dram__bytes_read+write of this format's kernels on this workload, hot reps (tools/traffic_corpus.py)
-        with open(os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json")) as fh:
+        with open(TRAFFIC_JSON) as fh:
             tj = json.load(fh).get(dom)
         if tj:
             traffic = tj["ratio"] * bytes_per_launch
             traffic_src = (f"ncu dram__bytes_read.sum + dram__bytes_write.sum of {tj['kernel']} over the corpus-200 race "
                            f"(last of 2 back-to-back calls per matrix, --cache-control none) = {tj['ratio']:.3f} x "
-                           f"the algorithmic bytes (profiles/r01/traffic_corpus200.json); < 1: the hot reps re-read "
+                           f"the algorithmic bytes ({os.path.relpath(TRAFFIC_JSON, ROOT)}); < 1: the hot reps re-read "
                            f"part of each matrix from L2")
     except Exception:
         pass
@@ -662,7 +665,7 @@ def run_ours(args):
     try:  # the L2-sector view: gather-heavy SpMVs are bound by the SM <- L2 sector rate, not by HBM
         with open(os.path.join(ROOT, "profiles", "r01", "ceilings.json")) as fh:
             cj = json.load(fh)
-        with open(os.path.join(ROOT, "profiles", "r01", "traffic_corpus200.json")) as fh:
+        with open(TRAFFIC_JSON) as fh:
             tj = json.load(fh).get(dom)
         if tj and tj.get("l2_sectors_per_launch"):
             rate = tj["l2_sectors_per_launch"] * launches_dom / per_fmt[dom]["spmv_time_s"] / 1e9
@@ -670,7 +673,7 @@ def run_ours(args):
                   "unit": "G sectors/s", "frac": rate / cj["l2_random_sector_rate_gsps"],
                   "sectors_per_launch": tj["l2_sectors_per_launch"],
                   "source": "ncu lts__t_sectors_srcunit_tex.sum of the same kernels on this workload "
-                            "(profiles/r01/traffic_corpus200.json) over this run's event-timed race time; peak = "
+                            f"({os.path.relpath(TRAFFIC_JSON, ROOT)}) over this run's event-timed race time; peak = "
                             "measured random-sector rate of tools/gather.cu (profiles/r01/ceilings.txt)"}
     except Exception:
         pass

@@ -26,10 +26,10 @@ def hyb_rowwise(f, z):
 
 def kernels_of(fmt, f, z):
     if fmt == 0:
-        if f["csr_variant"] in (3, 4) and z == 0:
+        if f["csr_variant"] in (3, 4, 5) and z == 0:
             return ["k_zero"]
         return {2: ["k_spmv_csr_stream"], 3: ["k_zero_rows", "k_spmv_csr_tile"],
-                4: ["k_zero_rows", "k_spmv_csr_tile"],
+                4: ["k_zero_rows", "k_spmv_csr_tile"], 5: ["k_zero", "k_spmv_csr_tile"],
                 1: ["k_spmv_csr_merge", "k_spmv_csr_merge_fixup"], 0: ["k_spmv_csr_vector"]}[f["csr_variant"]]
     if fmt == 1:
         return ["k_zero", "k_spmv_coo"]
