@@ -101,21 +101,6 @@ int grid_cap(long long items, int threads, int per_sm) {
   return (int)(g > cap ? cap : (g < 1 ? 1 : g));
 }
 
-// Grid of a grid-stride kernel over `items` work units with at most `cap` resident CTAs: every CTA gets
-// the same number of units (ceil(items / cap)), so the last round has no partial wave -- e.g. 2048
-// row blocks over 592 slots run as 512 CTAs x 4 blocks instead of 592 CTAs x 3.46 (a 13 % tail).
-// SFS_BALANCED_GRID=0: plain min(items, cap) (A/B).
-int balanced_grid(long long items, long long cap) {
-  static const bool on = [] {
-    const char* e = getenv("SFS_BALANCED_GRID");
-    return !(e && e[0] == '0');
-  }();
-  if (items <= cap) return (int)(items < 1 ? 1 : items);
-  if (!on) return (int)cap;
-  const long long per = ceil_div(items, cap);
-  return (int)ceil_div(items, per);
-}
-
 [[maybe_unused]] int pow2_ceil(long long v) {
   int p = 1;
   while (p < v && p < (1 << 20)) p <<= 1;
@@ -1435,7 +1420,7 @@ cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s,
   const long long groups = A->pitch / 4;
   const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
   const long long niter = ceil_div(groups, kEllThreads / S);
-  const int grid = balanced_grid(niter, (long long)kSMs * ell_ctas<T>());
+  const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
   if (!PUSH && A->fmt == SFS_HYB && A->variant == 1)
     return launch_k(k_spmv_ell<T, true, false>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
                     (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3],
@@ -1452,7 +1437,7 @@ cudaError_t launch_csr_stream(const int* rp, const int* col, const T* val, const
   const long long windows = ceil_div(z, 32 * stream_u<T>());  // ~ windows over all groups
   const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
   const long long niter = ceil_div(groups, kSWarps / S);
-  const int grid = balanced_grid(niter, (long long)kSMs * stream_ctas<T>());
+  const int grid = (int)(niter < (long long)kSMs * stream_ctas<T>() ? niter : (long long)kSMs * stream_ctas<T>());
   return launch_k(k_spmv_csr_stream<T, PUSH>, dim3(grid < 1 ? 1 : grid), dim3(kSThreads), s, rp, col, val, x, y, m, S,
                   push);
 }
@@ -1487,7 +1472,7 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   }();
   if (force_s == 1 || force_s == 2 || force_s == 4 || force_s == 8 || force_s == 16) S = force_s;
   const long long nblk = ceil_div(m, (long long)(kDiaThreads / S) * dia_rows<T>());
-  const int grid = balanced_grid(nblk, (long long)kSMs * dia_ctas<T>());
+  const int grid = (int)(nblk < (long long)kSMs * dia_ctas<T>() ? nblk : (long long)kSMs * dia_ctas<T>());
   const dim3 gd(grid < 1 ? 1 : grid), bd(kDiaThreads);
   const int* offs = (const int*)A->ptr[0];
   const T* dv = (const T*)A->ptr[1];
@@ -1583,7 +1568,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const long long windows = ceil_div(z, 32 * stream_u<T>());  // ~ windows over all groups
         const int S = split_factor(groups * 32, ceil_div(windows, groups), 1, kSWarps);
         const long long niter = ceil_div(groups, kSWarps / S);
-        const int grid = balanced_grid(niter, (long long)kSMs * stream_ctas<T>());
+        const int grid = (int)(niter < (long long)kSMs * stream_ctas<T>() ? niter : (long long)kSMs * stream_ctas<T>());
         e = launch_csr_stream<T, false>(rp, col, val, x, y, m, z, s, PushParam<false>{});
       } else if (A->variant == 0) {
         // kCsrWarps warps grid-stride over rows (the mapping the csr_max feature describes, Q4); a
