@@ -584,6 +584,9 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
 // the first chunk's loads and x gathers overlap it; the kernel waits before touching y.  No full zero
 // pass, no row array: CSR's own bytes only.
 constexpr int kTThreads = 256;
+#ifndef SFS_TILE_CTAS
+#define SFS_TILE_CTAS 4  // CTAs per SM of the tile kernel (register cap; A/B builds set 5)
+#endif
 constexpr int kTV = 8;
 constexpr int kTChunk = 32 * kTV;
 
@@ -593,7 +596,7 @@ struct TileGeom {
 TileGeom tile_geom(long long z) {
   TileGeom g;
   g.nchunks = ceil_div(z, kTChunk);
-  const long long max_warps = (long long)kSMs * 4 * (kTThreads / 32);  // one resident wave at 4 CTAs / SM
+  const long long max_warps = (long long)kSMs * SFS_TILE_CTAS * (kTThreads / 32);  // one resident wave
   g.cpw = ceil_div(g.nchunks, max_warps) < 1 ? 1 : ceil_div(g.nchunks, max_warps);
   g.nwarps = ceil_div(g.nchunks, g.cpw);
   return g;
@@ -800,7 +803,7 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
 
 // blockDim is 64, 128 or 256 (smaller CTAs spread a small matrix's few warps over more SMs)
 template <typename T, bool VEC, bool BM, bool MAP = false>
-__global__ void __launch_bounds__(kTThreads, 4) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
+__global__ void __launch_bounds__(kTThreads, SFS_TILE_CTAS) k_spmv_csr_tile(const int* __restrict__ rp, const int* __restrict__ col,
                                                                const T* __restrict__ val, const T* __restrict__ x,
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
@@ -1239,15 +1242,21 @@ __global__ void __launch_bounds__(kDiaThreads, dia_ctas<T>()) k_spmv_dia(const i
 // (the ELL mapping; warp = 128 consecutive rows, 512 contiguous bytes per slab load) and its 4 x values
 // are 4 scalar loads hitting the same lines (L1).  fp32's scalar strided mapping above moves 4 bytes
 // per load instruction; this one moves 16.  S diagonal-parts per row block meet in shared memory.
+#ifndef SFS_DIA_V4_CTAS
+#define SFS_DIA_V4_CTAS 4  // CTAs per SM (register cap); A/B builds set 5 / 6 together with SFS_DIA_V4_KB
+#endif
+#ifndef SFS_DIA_V4_KB
+#define SFS_DIA_V4_KB 4    // fp32 diagonals per batch
+#endif
 template <typename T, int S, bool PUSH, bool XA = false>
-__global__ void __launch_bounds__(kDiaThreads, 4) k_spmv_dia_v4(const int* __restrict__ offs,
+__global__ void __launch_bounds__(kDiaThreads, SFS_DIA_V4_CTAS) k_spmv_dia_v4(const int* __restrict__ offs,
                                                                 const T* __restrict__ dval,
                                                                 const T* __restrict__ x, T* __restrict__ y,
                                                                 long long m, long long n, long long P, int nd,
                                                                 PushParam<PUSH> push, int pfd) {
   static_assert(!XA || sizeof(T) == 4, "XA: fp32 x");
   constexpr int G = kDiaThreads / S;
-  constexpr int kB = sizeof(T) == 4 ? 4 : 2;  // diagonals per batch (register cap)
+  constexpr int kB = sizeof(T) == 4 ? SFS_DIA_V4_KB : 2;  // diagonals per batch (register cap)
   __shared__ int s_off[kDiaSmemOffs];
   __shared__ acc_t s_part[S > 1 ? kDiaThreads * 4 : 1];
   pdl_wait();
@@ -1485,6 +1494,8 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
       return e ? atoi(e) : 1;
     }();
     // same split rule; 4 consecutive rows per thread (G * 4 rows per block, as the strided mapping)
+    const int g4 = (int)(nblk < (long long)kSMs * SFS_DIA_V4_CTAS ? nblk : (long long)kSMs * SFS_DIA_V4_CTAS);
+    const dim3 gd(g4 < 1 ? 1 : g4);
     if constexpr (sizeof(T) == 4) {
       static const bool xa = [] {  // SFS_DIA_XA=0: 4 scalar x loads per diagonal (A/B)
         const char* e = getenv("SFS_DIA_XA");
