@@ -883,7 +883,10 @@ __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
   else y[row] = (T)v;
 }
 
-template <typename T, bool ACCUM>
+// ATOM (the COO part of an overlapped HYB): y was zeroed before the ELL part, which runs concurrently and
+// adds atomically -- every row sum is added atomically too, nothing waits before touching y, and the grid
+// waits for its predecessor (the ELL part) only at its end, so the SpMV is complete when this grid is.
+template <typename T, bool ACCUM, bool ATOM = false>
 __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
                                                           T* __restrict__ y, long long z, long long chunks_per_warp) {
@@ -928,7 +931,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
           }
         }
       }
-      if (!waited) {
+      if (!ATOM && !waited) {
         pdl_wait();
         pdl_early();
         waited = true;
@@ -937,7 +940,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       // the previous chunk's carry ends exactly at this chunk boundary: emit it
       const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
       if (carry_row >= 0 && carry_row != chunk_first) {
-        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, carry_row == range_first);
+        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, ATOM || carry_row == range_first);
         carry_row = -1;
         carry = 0;
       }
@@ -949,7 +952,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       for (int i = 1; i < kCooV; i++) {
         if (r[i] != cr) {
           if (in_head) { head = cur; in_head = false; }
-          else coo_emit<T, ACCUM>(y, cr, cur, cr == range_first);
+          else coo_emit<T, ACCUM>(y, cr, cur, ATOM || cr == range_first);
           cr = r[i];
           cur = p[i];
         } else {
@@ -976,15 +979,17 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
       if (!single) {
         const acc_t h = head + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0)));
-        coo_emit<T, ACCUM>(y, rf, h, rf == range_first);
+        coo_emit<T, ACCUM>(y, rf, h, ATOM || rf == range_first);
       }
-      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, rl == range_first);
+      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, ATOM || rl == range_first);
       carry_row = __shfl_sync(0xffffffffu, rl, 31);  // the chunk's last row stays open
       carry = __shfl_sync(0xffffffffu, S, 31);
     }
     if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
   }
-  if (!waited) pdl_wait();
+  // ATOM: complete only after the ELL part (its predecessor) has completed, so the SpMV is done with this
+  // grid and the next SpMV's zero kernel cannot overtake the ELL part's atomics
+  if (ATOM || !waited) pdl_wait();
   pdl_trigger();
 }
 
@@ -1002,7 +1007,9 @@ template <typename T> constexpr int ell_ctas() { return sizeof(T) == 4 ? 3 : 4; 
 constexpr long long kHybRowwiseSmall = 64;  // z < 2^20 (latency-bound sizes)
 constexpr long long kHybRowwiseLarge = 32;
 
-template <typename T, bool OVF, bool PUSH = false>
+// ATOM (HYB with long overflow rows, overlapped): y was zeroed ahead and the COO part runs concurrently,
+// so the ELL part adds its row sums atomically instead of storing them.
+template <typename T, bool OVF, bool PUSH = false, bool ATOM = false>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
                                                                          const T* __restrict__ eval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
@@ -1122,8 +1129,12 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
     }
     if (p == 0 && grp < groups) {
 #pragma unroll
-      for (int q = 0; q < 4; q++)
-        if (r + q < m) store_row<PUSH>(y, r + q, (T)acc[q], push, pushed);
+      for (int q = 0; q < 4; q++) {
+        if (r + q < m) {
+          if constexpr (ATOM) atomicAdd(y + r + q, (T)acc[q]);
+          else store_row<PUSH>(y, r + q, (T)acc[q], push, pushed);
+        }
+      }
     }
   }
   halo_signal<PUSH>(push, pushed);
@@ -1408,14 +1419,14 @@ TileWork tile_work(void* base, const TileGeom& g) {
 }
 
 // COO launch geometry: contiguous chunk ranges, one resident wave of warps at most.
-template <typename T, bool ACCUM>
+template <typename T, bool ACCUM, bool ATOM = false>
 cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
   const long long nchunks = ceil_div(z, kChunk);
   const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);  // <= 64 regs: 4 CTAs / SM
   const long long cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
   const long long warps = ceil_div(nchunks, cpw);
   const unsigned blocks = (unsigned)ceil_div(warps, kCooThreads / 32);
-  return launch_k(k_spmv_coo<T, ACCUM>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
+  return launch_k(k_spmv_coo<T, ACCUM, ATOM>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
 }
 
 template <typename T>
@@ -1423,7 +1434,7 @@ cudaError_t launch_zero(T* y, long long m, cudaStream_t s) {
   return launch_k(k_zero<T>, dim3(grid_cap(m, 256, 8)), dim3(256), s, y, m);
 }
 
-template <typename T, bool PUSH = false>
+template <typename T, bool PUSH = false, bool ATOM = false>
 cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s, int early_trigger,
                        PushParam<PUSH> push = {}) {
   const long long groups = A->pitch / 4;
@@ -1434,7 +1445,7 @@ cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s,
     return launch_k(k_spmv_ell<T, true, false>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
                     (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3],
                     (const T*)A->ptr[4], PushParam<false>{});
-  return launch_k(k_spmv_ell<T, false, PUSH>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
+  return launch_k(k_spmv_ell<T, false, PUSH, ATOM>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
                   (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, early_trigger, (const int*)nullptr,
                   (const int*)nullptr, (const T*)nullptr, push);
 }
@@ -1528,6 +1539,15 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   }
 }
 
+// HYB with long overflow rows: overlapped parts (SFS_HYB_OVERLAP=0: the ELL part -> COO<ACCUM> pair)
+bool hyb_overlap() {
+  static const bool v = [] {
+    const char* e = getenv("SFS_HYB_OVERLAP");
+    return !(e && e[0] == '0');
+  }();
+  return v;
+}
+
 template <typename T>
 cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
   const long long m = A->m, z = A->nnz;
@@ -1615,6 +1635,16 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
     case SFS_HYB: {
       const int K = (int)A->width;
       const bool two = A->fmt == SFS_HYB && A->coo_nnz > 0 && A->variant == 0;  // ELL part -> COO part
+      if (two && K > 0 && hyb_overlap()) {
+        // zero -> ELL part (atomic adds, releases the COO part at its start) -> COO part (atomic adds,
+        // waits for the ELL part only before it exits): the two parts run concurrently
+        e = launch_zero<T>(y, m, s);
+        if (e == cudaSuccess) e = launch_ell<T, false, true>(A, x, y, K, s, 1);
+        if (e == cudaSuccess)
+          e = launch_coo<T, true, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y,
+                                        A->coo_nnz, s);
+        break;
+      }
       e = K == 0 ? launch_zero<T>(y, m, s) : launch_ell<T>(A, x, y, K, s, two);
       if (e == cudaSuccess && two)
         e = launch_coo<T, true>((const int*)A->ptr[2], (const int*)A->ptr[3], (const T*)A->ptr[4], x, y, A->coo_nnz, s);
@@ -1734,7 +1764,7 @@ int spmv_kernels_per_call(const Matrix* A) {
   switch (A->fmt) {
     case SFS_CSR: return (A->variant == 1 || ((A->variant >= 3 && A->variant <= 5) && A->nnz > 0)) ? 2 : 1;
     case SFS_COO: return A->nnz > 0 ? 2 : 1;
-    case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? 2 : 1;
+    case SFS_HYB: return (A->coo_nnz > 0 && A->variant == 0) ? (A->width > 0 && hyb_overlap() ? 3 : 2) : 1;
     default: return 1;
   }
 }
