@@ -40,7 +40,7 @@ def kernels_of(fmt, f, z):
             return ["k_zero", "k_spmv_coo"]
         if f["hyb_coo"] == 0 or hyb_rowwise(f, z):
             return ["k_spmv_ell"]
-        return ["k_spmv_ell", "k_spmv_coo"]
+        return ["k_zero", "k_spmv_ell", "k_spmv_coo"]  # overlapped parts
     return ["k_spmv_dia"]
 
 
