@@ -338,15 +338,6 @@ static sfs_status features_finish(const DevCSR& d, const sfs_race_opts& o, const
   return SFS_OK;
 }
 
-// SFS_COO_SPLIT_ZERO=0: COO always clears all of y ahead of its kernel (A/B switch)
-static bool coo_split_zero() {
-  static const bool v = [] {
-    const char* e = getenv("SFS_COO_SPLIT_ZERO");
-    return !(e && e[0] == '0');
-  }();
-  return v;
-}
-
 // ---------------------------------------------------------------- conversion
 static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_features_t& f, const FeatWork& fw,
                                Matrix** out, cudaStream_t s) {
@@ -420,11 +411,6 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
       if (!r || !c || !v) return bail(SFS_ERR_OOM, "coo");
       BAIL_CUDA(launch_csr2coo(d.dtype, d.rp, d.col, d.val, m, z, r, c, v, s));
       A->ptr[0] = r; A->ptr[1] = c; A->ptr[2] = v;
-      if (z > 0 && f.nnz_min >= 1 && coo_split_zero()) {  // every row holds an entry: clear only split rows
-        A->work = own(coo_split_work_bytes(z));
-        if (!A->work) return bail(SFS_ERR_OOM, "coo split rows");
-        BAIL_CUDA(launch_coo_split_prepare(r, m, z, A->work, s));
-      }
       break;
     }
     case SFS_ELL: {

@@ -104,9 +104,6 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap);
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s);
 int csr_vector_tpv(long long m, long long z);
-// COO of a matrix without empty rows: the split rows at warp-range boundaries (cleared ahead of the SpMV)
-size_t coo_split_work_bytes(long long z);
-cudaError_t launch_coo_split_prepare(const int* row, long long m, long long z, void* work, cudaStream_t s);
 int hyb_rowwise(long long nnz_max, long long K, long long coo_nnz, long long z);
 cudaError_t launch_fill(int dtype, void* p, long long n, double v, cudaStream_t s);
 // dst[i] = src[idx[i]], i < n (exchange.cu: halo send buffers of the row-partitioned SpMV)
@@ -139,7 +136,7 @@ struct Matrix {
   int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile, 4 tile + row-start bitmap,
                                // 5 tile + bitmap over the non-empty rows + row map;
                                // HYB: 1 = one launch (ptr[5] = ovf)
-  void* work = nullptr;        // CSR merge / tile partition and carries; COO split-row list (no empty row)
+  void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;
   void (*user_free)(void*, void*) = nullptr;  // allocator hook at creation (nullptr: the library's pool)
 };

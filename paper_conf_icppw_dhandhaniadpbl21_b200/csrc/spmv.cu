@@ -886,11 +886,7 @@ __device__ __forceinline__ void coo_emit(T* y, int row, acc_t v, bool atomic) {
 // ATOM (the COO part of an overlapped HYB): y was zeroed before the ELL part, which runs concurrently and
 // adds atomically -- every row sum is added atomically too, nothing waits before touching y, and the grid
 // waits for its predecessor (the ELL part) only at its end, so the SpMV is complete when this grid is.
-// SPLITZ (COO of a matrix without empty rows): only the rows split across warp ranges were zeroed ahead
-// (k_zero_rows over the handle's split-row list instead of a pass over all of y); a range's first row is
-// added atomically only if it started in the previous range, its final carry only if the row continues
-// into the next range, every other row is stored.
-template <typename T, bool ACCUM, bool ATOM = false, bool SPLITZ = false>
+template <typename T, bool ACCUM, bool ATOM = false>
 __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict__ row, const int* __restrict__ col,
                                                           const T* __restrict__ val, const T* __restrict__ x,
                                                           T* __restrict__ y, long long z, long long chunks_per_warp) {
@@ -905,9 +901,6 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
   if (cb < ce) {
     const int last_row = __ldg(row + z - 1);
     const int range_first = __ldg(row + cb * kChunk);
-    // SPLITZ: is range_first split (started before this range)?  Does the last row continue after it?
-    const bool first_split = !SPLITZ || (cb > 0 && __ldg(row + cb * kChunk - 1) == range_first);
-    const int next_first = SPLITZ && ce < nchunks ? __ldg(row + ce * kChunk) : -1;
     int carry_row = -1;
     acc_t carry = 0;
     for (long long ch = cb; ch < ce; ch++) {
@@ -947,7 +940,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       // the previous chunk's carry ends exactly at this chunk boundary: emit it
       const int chunk_first = __shfl_sync(0xffffffffu, rf, 0);
       if (carry_row >= 0 && carry_row != chunk_first) {
-        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, ATOM || (carry_row == range_first && first_split));
+        if (l == 0) coo_emit<T, ACCUM>(y, carry_row, carry, ATOM || carry_row == range_first);
         carry_row = -1;
         carry = 0;
       }
@@ -959,7 +952,7 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       for (int i = 1; i < kCooV; i++) {
         if (r[i] != cr) {
           if (in_head) { head = cur; in_head = false; }
-          else coo_emit<T, ACCUM>(y, cr, cur, ATOM || (cr == range_first && first_split));
+          else coo_emit<T, ACCUM>(y, cr, cur, ATOM || cr == range_first);
           cr = r[i];
           cur = p[i];
         } else {
@@ -986,18 +979,13 @@ __global__ void __launch_bounds__(kCooThreads) k_spmv_coo(const int* __restrict_
       const int next_rf = __shfl_down_sync(0xffffffffu, rf, 1);
       if (!single) {
         const acc_t h = head + (l == 0 ? in0 : (prev_rl == rf ? S_prev : acc_t(0)));
-        coo_emit<T, ACCUM>(y, rf, h, ATOM || (rf == range_first && first_split));
+        coo_emit<T, ACCUM>(y, rf, h, ATOM || rf == range_first);
       }
-      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, ATOM || (rl == range_first && first_split));
+      if (l < 31 && next_rf != rl) coo_emit<T, ACCUM>(y, rl, S, ATOM || rl == range_first);
       carry_row = __shfl_sync(0xffffffffu, rl, 31);  // the chunk's last row stays open
       carry = __shfl_sync(0xffffffffu, S, 31);
     }
-    if (l == 0 && carry_row >= 0) {  // may continue in the next range
-      if (SPLITZ && carry_row != next_first && !(carry_row == range_first && first_split))
-        coo_emit<T, ACCUM>(y, carry_row, carry, false);  // ends with the range, not split: a plain store
-      else
-        atomicAdd(y + carry_row, (T)carry);
-    }
+    if (l == 0 && carry_row >= 0) atomicAdd(y + carry_row, (T)carry);  // may continue in the next range
   }
   // ATOM: complete only after the ELL part (its predecessor) has completed, so the SpMV is done with this
   // grid and the next SpMV's zero kernel cannot overtake the ELL part's atomics
@@ -1430,31 +1418,15 @@ TileWork tile_work(void* base, const TileGeom& g) {
   return w;
 }
 
-// COO split rows (no empty row): srow[w] = the row of warp w's first entry if it started in an earlier
-// range, else m -- the rows k_zero_rows clears ahead of the SPLITZ kernel
-long long coo_cpw(long long z) {
-  const long long nchunks = ceil_div(z, kChunk);
-  const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);
-  return ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
-}
-long long coo_warps(long long z) { return ceil_div(ceil_div(z, kChunk), coo_cpw(z)); }
-__global__ void k_coo_split_rows(const int* __restrict__ row, long long z, long long cpw, long long nwarps, long long m,
-                                 int* __restrict__ srow) {
-  for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nwarps; w += (long long)gridDim.x * blockDim.x) {
-    const long long k = w * cpw * kChunk;
-    srow[w] = (w > 0 && k < z && row[k - 1] == row[k]) ? row[k] : (int)m;
-  }
-}
-
 // COO launch geometry: contiguous chunk ranges, one resident wave of warps at most.
-template <typename T, bool ACCUM, bool ATOM = false, bool SPLITZ = false>
+template <typename T, bool ACCUM, bool ATOM = false>
 cudaError_t launch_coo(const int* row, const int* col, const T* val, const T* x, T* y, long long z, cudaStream_t s) {
   const long long nchunks = ceil_div(z, kChunk);
   const long long max_warps = (long long)kSMs * 4 * (kCooThreads / 32);  // <= 64 regs: 4 CTAs / SM
   const long long cpw = ceil_div(nchunks, max_warps) < 1 ? 1 : ceil_div(nchunks, max_warps);
   const long long warps = ceil_div(nchunks, cpw);
   const unsigned blocks = (unsigned)ceil_div(warps, kCooThreads / 32);
-  return launch_k(k_spmv_coo<T, ACCUM, ATOM, SPLITZ>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
+  return launch_k(k_spmv_coo<T, ACCUM, ATOM>, dim3(blocks), dim3(kCooThreads), s, row, col, val, x, y, z, cpw);
 }
 
 template <typename T>
@@ -1654,14 +1626,6 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
       break;
     }
     case SFS_COO: {
-      if (A->work && z > 0) {  // no empty row: zero only the split rows (srow list built with the handle)
-        const long long nw = coo_warps(z);
-        e = launch_k(k_zero_rows<T>, dim3(grid_cap(nw, 256, 4)), dim3(256), s, y, (const int*)A->work, nw, m);
-        if (e == cudaSuccess)
-          e = launch_coo<T, false, false, true>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x,
-                                               y, z, s);
-        break;
-      }
       e = launch_zero<T>(y, m, s);
       if (e == cudaSuccess && z > 0)
         e = launch_coo<T, false>((const int*)A->ptr[0], (const int*)A->ptr[1], (const T*)A->ptr[2], x, y, z, s);
@@ -1712,15 +1676,6 @@ __global__ void k_fill(T* __restrict__ p, long long n, T v) {
 }
 
 }  // namespace
-
-size_t coo_split_work_bytes(long long z) { return al256(sizeof(int) * coo_warps(z)); }
-
-cudaError_t launch_coo_split_prepare(const int* row, long long m, long long z, void* work, cudaStream_t s) {
-  const long long nw = coo_warps(z);
-  k_coo_split_rows<<<grid_cap(nw, 256, 8), 256, 0, s>>>(row, z, coo_cpw(z), nw, m, (int*)work);
-  count_launch();
-  return cudaGetLastError();
-}
 
 int csr_vector_tpv(long long m, long long z) {
   const long long avg = z / m;
