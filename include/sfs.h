@@ -147,7 +147,8 @@ sfs_status sfs_convert(const sfs_csr *A, sfs_format f, const sfs_race_opts *opt,
 
 /* y = A·x with A in format f (f must equal A's format, else INVALID_ARG).  x has ncols
    entries, y has nrows entries, device pointers of A's dtype; y is fully overwritten.  Asynchronous:
-   1–2 kernel launches on `stream`, no synchronization. */
+   1–3 kernel launches on `stream` (a zero pass and the kernels of the format; HYB with long overflow
+   rows runs its ELL and COO parts concurrently), no synchronization. */
 sfs_status sfs_spmv(sfs_format f, sfs_matrix A, const void *x, void *y, void *stream);
 
 /* Label a batch of matrices: features of all n matrices (batched), then for each
