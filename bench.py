@@ -642,9 +642,11 @@ def run_ours(args):
     peak_src = "measured (MEASURED_PEAKS.json hbm_gbs)"
     if not peak:
         peak, peak_src = 6650.0, "fallback (B200_PROFILING.md)"
-    kernels = {"CSR": "k_spmv_csr_tile<bitmap> + fixup (large or skewed, no empty rows) / k_spmv_csr_stream "
-                      "(small regular) / k_spmv_csr_merge + fixup (many empty rows)",
-               "COO": "k_zero + k_spmv_coo", "ELL": "k_spmv_ell", "HYB": "k_spmv_ell + k_spmv_coo<ACCUM>",
+    kernels = {"CSR": "k_zero_rows + k_spmv_csr_tile<bitmap> (large or skewed) / k_spmv_csr_stream (small regular) / "
+                      "k_zero + k_spmv_csr_tile<bitmap, row map> (empty rows)",
+               "COO": "k_zero + k_spmv_coo", "ELL": "k_spmv_ell",
+               "HYB": "k_spmv_ell<OVF> (short overflow) / k_zero + k_spmv_ell<ATOM> || k_spmv_coo<ACCUM,ATOM> "
+                      "(long overflow, parts overlapped)",
                "DIA": "k_spmv_dia"}
     achieved = per_fmt[dom]["gbs"]
     launches_dom = sum(1 for L in labs if L["status"][sfs.FORMAT_NAMES.index(dom)] == 0) * args.reps
