@@ -1009,9 +1009,7 @@ constexpr long long kHybRowwiseLarge = 32;
 
 // ATOM (HYB with long overflow rows, overlapped): y was zeroed ahead and the COO part runs concurrently,
 // so the ELL part adds its row sums atomically instead of storing them.
-// LP: the S slot-parts of a row group are S lanes of one warp (lane & (S-1)) instead of S warps, so
-// the parts meet through warp shuffles and no CTA barrier is needed per row-group round.
-template <typename T, bool OVF, bool PUSH = false, bool ATOM = false, bool LP = false>
+template <typename T, bool OVF, bool PUSH = false, bool ATOM = false>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
                                                                          const T* __restrict__ eval,
                                                                          const T* __restrict__ x, T* __restrict__ y,
@@ -1022,22 +1020,14 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
                                                                          const T* __restrict__ oval,
                                                                          PushParam<PUSH> push) {
   constexpr int kB = ell_batch<T>();
-  __shared__ acc_t s_part[LP ? 1 : kEllThreads][4];
+  __shared__ acc_t s_part[kEllThreads][4];
   pdl_wait();
   pdl_early();
   if (early_trigger) pdl_trigger();  // HYB: let the COO part start its loads now
   halo_wait<PUSH>(push);
   bool pushed = false;
   const int G = kEllThreads / S;
-  int p, g;
-  if constexpr (LP) {
-    const int sh = __ffs(S) - 1, lane = threadIdx.x & 31;
-    p = lane & (S - 1);
-    g = (threadIdx.x >> 5) * (32 >> sh) + (lane >> sh);
-  } else {
-    p = threadIdx.x / G;
-    g = threadIdx.x % G;
-  }
+  const int p = threadIdx.x / G, g = threadIdx.x % G;
   const int Kp = (K + S - 1) / S;
   const int j0 = p * Kp, j1 = j0 + Kp < K ? j0 + Kp : K;
   const long long groups = P / 4;
@@ -1126,11 +1116,7 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
         }
       }
     }
-    if constexpr (LP) {
-      for (int o = 1; o < S; o <<= 1)
-#pragma unroll
-        for (int q = 0; q < 4; q++) acc[q] += __shfl_xor_sync(0xffffffffu, acc[q], o);
-    } else if (S > 1) {
+    if (S > 1) {
 #pragma unroll
       for (int q = 0; q < 4; q++) s_part[threadIdx.x][q] = acc[q];
       __syncthreads();
@@ -1448,15 +1434,6 @@ cudaError_t launch_zero(T* y, long long m, cudaStream_t s) {
   return launch_k(k_zero<T>, dim3(grid_cap(m, 256, 8)), dim3(256), s, y, m);
 }
 
-// SFS_ELL_LP=0: the slot-parts of a row group in different warps, met in shared memory (A/B)
-bool ell_lane_parts() {
-  static const bool v = [] {
-    const char* e = getenv("SFS_ELL_LP");
-    return !(e && e[0] == '0');
-  }();
-  return v;
-}
-
 template <typename T, bool PUSH = false, bool ATOM = false>
 cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s, int early_trigger,
                        PushParam<PUSH> push = {}) {
@@ -1464,8 +1441,7 @@ cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s,
   const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
   const long long niter = ceil_div(groups, kEllThreads / S);
   const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
-  if (S > 1 && ell_lane_parts()) {
-    if (!PUSH && A->fmt == SFS_HYB && A->variant == 1)
+  if (!PUSH && A->fmt == SFS_HYB && A->variant == 1)
       return launch_k(k_spmv_ell<T, true, false, false, true>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
                       (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3],
                       (const T*)A->ptr[4], PushParam<false>{});
