@@ -1442,14 +1442,6 @@ cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s,
   const long long niter = ceil_div(groups, kEllThreads / S);
   const int grid = (int)(niter < (long long)kSMs * ell_ctas<T>() ? niter : (long long)kSMs * ell_ctas<T>());
   if (!PUSH && A->fmt == SFS_HYB && A->variant == 1)
-      return launch_k(k_spmv_ell<T, true, false, false, true>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
-                      (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3],
-                      (const T*)A->ptr[4], PushParam<false>{});
-    return launch_k(k_spmv_ell<T, false, PUSH, ATOM, true>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
-                    (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, early_trigger, (const int*)nullptr,
-                    (const int*)nullptr, (const T*)nullptr, push);
-  }
-  if (!PUSH && A->fmt == SFS_HYB && A->variant == 1)
     return launch_k(k_spmv_ell<T, true, false>, dim3(grid), dim3(kEllThreads), s, (const int*)A->ptr[0],
                     (const T*)A->ptr[1], x, y, A->m, A->pitch, K, S, 0, (const int*)A->ptr[5], (const int*)A->ptr[3],
                     (const T*)A->ptr[4], PushParam<false>{});
