@@ -32,6 +32,8 @@
 #include <stdlib.h>
 
 #include <algorithm>
+#include <mutex>
+#include <type_traits>
 
 #include "common.cuh"
 #include "internal.h"
@@ -86,6 +88,22 @@ cudaError_t launch_k(void (*kern)(Params...), dim3 grid, dim3 block, cudaStream_
   cfg.gridDim = grid;
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  count_launch();
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<Params>(args)...);
+}
+
+template <typename... Params, typename... Args>
+cudaError_t launch_k_smem(void (*kern)(Params...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
   cfg.stream = s;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -1382,6 +1400,256 @@ __global__ void __launch_bounds__(kDiaThreads, SFS_DIA_V4_CTAS) k_spmv_dia_v4(co
   pdl_trigger();
 }
 
+// Shared by the TMA DIA kernel below: rows per block, staged-x window rules, cp.async helpers.
+constexpr int kSxRows = 4 * kDiaThreads;  // rows per block: thread t owns rows t + 256 q, q = 0..3
+constexpr int kSxBuf = 16384;             // bytes per fp32 x staging buffer (two per CTA)
+constexpr int kSxGap = 256;               // offsets closer than this share an x window
+constexpr int kSxWin = 32;                // windows tracked (later ones read x from global memory)
+__device__ __forceinline__ void cp_async16(void* dst, const void* src, int src_bytes) {
+  const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(d), "l"(src), "r"(src_bytes) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
+
+// Window setup of the staged-x DIA kernel (warp 0; the caller synchronises): offsets closer than kSxGap
+// share a window; window w (w < kSxWin) holds (whi - floor4(wlo)) + kSxRows values rounded up to 4 at
+// s_wsb[w]; staged windows are the prefix that fits kCap values.  s_xb[d] = window of d (-1: none).
+__device__ __forceinline__ void sx_windows(int nd, int kCap, const int* s_off, int* s_xb, int* s_wlo, int* s_whi,
+                                           int* s_wlen, int* s_wsb, int* s_nw, int* s_tot, int* s_all) {
+  const int lane = threadIdx.x & 31;
+  {
+    int nw = 0;
+    for (int d0 = 0; d0 < nd; d0 += 32) {
+      const int d = d0 + lane;
+      const bool ok = d < nd;
+      const int o = ok ? s_off[d] : 0;
+      const bool start = ok && (d == 0 || o - s_off[d - 1] > kSxGap);
+      const bool end = ok && (d == nd - 1 || s_off[d + 1] - o > kSxGap);
+      const unsigned sb = __ballot_sync(0xffffffffu, start);
+      const int w = nw + __popc(sb & ((2u << lane) - 1u)) - 1;  // window of d
+      if (ok) s_xb[d] = w < kSxWin ? w : -1;
+      if (start && w < kSxWin) s_wlo[w] = o;
+      if (end && w < kSxWin) s_whi[w] = o;
+      nw += __popc(sb);
+    }
+    const bool fits = nw <= kSxWin;
+    nw = nw < kSxWin ? nw : kSxWin;
+    __syncwarp();
+    // budget: window w holds (whi - floor4(wlo)) + kSxRows values rounded up to 4; staged windows are a
+    // prefix (the running total is monotone)
+    int len = 0;
+    if (lane < nw) len = ((s_whi[lane] - (s_wlo[lane] & ~3) + kSxRows) + 3) & ~3;
+    int inc = len;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int u = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += u;
+    }
+    const bool staged = lane < nw && inc <= kCap;
+    if (lane < nw) {
+      s_wlen[lane] = staged ? len : 0;
+      s_wsb[lane] = inc - len;
+    }
+    const int ns = __popc(__ballot_sync(0xffffffffu, staged));
+    const int tot = __shfl_sync(0xffffffffu, inc, ns > 0 ? ns - 1 : 0);  // values staged per block
+    if (lane == 0) {
+      *s_nw = ns;
+      *s_tot = ns > 0 ? tot : 0;
+      *s_all = fits && ns == nw;  // every diagonal's x is staged
+    }
+  }
+}
+
+// DIA with the slab streamed by TMA bulk copies (cp.async.bulk) through a ring of shared-memory stages and
+// x staged as in k_spmv_dia_sx (large matrices).  A producer warp issues, per (row block, batch of kTB
+// diagonals), one bulk copy of each diagonal's kSxRows-row slab segment (contiguous: the slab is
+// diagonal-major) into a free stage and arms that stage's mbarrier with the byte count; the 8 consumer
+// warps wait on the stage's mbarrier, read slab and x from shared memory (thread t: rows t + 256 q, both
+// reads conflict-free), and release the stage to the producer through a second mbarrier.  The bytes in
+// flight per SM are the ring (kTStages x kTB x 4 KB per CTA), held by no register -- the limit of the
+// register-staged fp32 kernels (latency-bound at ~0.73-0.79 of HBM).  x windows: cp.async by the
+// consumers, double-buffered per block, synchronised by a consumer-only named barrier.
+// ring depth (measured, cold, tools/micro.py: fp32 4 stages at 2 CTAs / SM -- 128^3 stencil 0.86 of HBM, 6 or
+// 8 stages at 1 CTA / SM 0.66-0.70; fp64 8 stages at 1 CTA / SM -- stencil 0.93, 1M-row band 0.92)
+#ifndef SFS_DIA_TMA_STAGES32
+#define SFS_DIA_TMA_STAGES32 4
+#endif
+#ifndef SFS_DIA_TMA_STAGES64
+#define SFS_DIA_TMA_STAGES64 8
+#endif
+template <typename T> constexpr int dia_tma_stages() { return sizeof(T) == 4 ? SFS_DIA_TMA_STAGES32 : SFS_DIA_TMA_STAGES64; }
+constexpr int kTConsumers = kDiaThreads;            // 8 consumer warps
+constexpr int kTThreadsAll = kDiaThreads + 32;      // + 1 producer warp
+template <typename T> constexpr int dia_tma_batch() { return 16384 / (kSxRows * (int)sizeof(T)); }  // 16 KB stages
+#ifndef SFS_DIA_TMA_XBUF64
+#define SFS_DIA_TMA_XBUF64 32768  // fp64 x buffer bytes (the 128^3 stencil's 3 windows need 30.9 KB)
+#endif
+template <typename T> constexpr int dia_tma_xbuf() { return sizeof(T) == 8 ? SFS_DIA_TMA_XBUF64 : kSxBuf; }
+template <typename T>
+constexpr size_t dia_tma_smem() {
+  return (size_t)dia_tma_stages<T>() * dia_tma_batch<T>() * kSxRows * sizeof(T) + 2 * (size_t)dia_tma_xbuf<T>();
+}
+__device__ __forceinline__ unsigned smem_u32(const void* p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned a, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(a), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned a, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n"
+      "WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}\n" ::"r"(a),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned a) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(a) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned a, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(a), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void tma_bulk_g2s(unsigned dst, const void* src, unsigned bytes, unsigned mbar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(mbar)
+               : "memory");
+}
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kTConsumers) : "memory"); }
+
+template <typename T>
+__global__ void __launch_bounds__(kTThreadsAll, 1) k_spmv_dia_tma(const int* __restrict__ offs, const T* __restrict__ dval,
+                                                                  const T* __restrict__ x, T* __restrict__ y,
+                                                                  long long m, long long n, long long P, int nd) {
+  constexpr int kB = dia_tma_batch<T>();
+  constexpr int kTStages = dia_tma_stages<T>();
+  constexpr int kCap = dia_tma_xbuf<T>() / (int)sizeof(T);
+  constexpr int kE = 16 / (int)sizeof(T);
+  extern __shared__ __align__(128) unsigned char s_dyn[];
+  T* s_slab = reinterpret_cast<T*>(s_dyn);                                       // [stage][u][row]
+  T* s_xbuf = reinterpret_cast<T*>(s_dyn + (size_t)kTStages * kB * kSxRows * sizeof(T));  // [2][kCap]
+  __shared__ __align__(8) unsigned long long s_full[16], s_empty[16];
+  __shared__ int s_off[kDiaSmemOffs];
+  __shared__ int s_xb[kDiaSmemOffs];
+  __shared__ int s_wlo[kSxWin], s_whi[kSxWin], s_wlen[kSxWin], s_wsb[kSxWin];
+  __shared__ int s_nw, s_tot, s_all;
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  if (t == 0) {
+    for (int i = 0; i < kTStages; i++) {
+      mbar_init(smem_u32(&s_full[i]), 1);
+      mbar_init(smem_u32(&s_empty[i]), kTConsumers / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  pdl_wait();
+  for (int i = t; i < nd; i += blockDim.x) s_off[i] = offs[i];
+  __syncthreads();
+  if (t < 32) sx_windows(nd, kCap, s_off, s_xb, s_wlo, s_whi, s_wlen, s_wsb, &s_nw, &s_tot, &s_all);
+  __syncthreads();
+  for (int d = t; d < nd; d += blockDim.x) {
+    const int w = s_xb[d];
+    s_xb[d] = (w >= 0 && s_wlen[w] > 0) ? s_wsb[w] + (s_off[d] - (s_wlo[w] & ~3)) : -1;
+  }
+  __syncthreads();
+  const long long nblk = ceil_div(m, (long long)kSxRows);
+  const int nbatch = (nd + kB - 1) / kB;
+  if (warp == kTConsumers / 32) {  // producer warp: one lane issues every bulk copy
+    if (lane == 0) {
+      long long i = 0;
+      for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const long long rbase = blk * kSxRows;
+        const long long rows = P - rbase < kSxRows ? P - rbase : kSxRows;  // P: multiple of 32, >= m
+        const unsigned seg = (unsigned)(rows * (long long)sizeof(T));
+        for (int b = 0; b < nbatch; b++, i++) {
+          const int st = (int)(i % kTStages);
+          const long long round = i / kTStages;
+          if (round > 0) mbar_wait(smem_u32(&s_empty[st]), (unsigned)((round - 1) & 1));
+          const int d0 = b * kB, nb = nd - d0 < kB ? nd - d0 : kB;
+          const unsigned full = smem_u32(&s_full[st]);
+          mbar_expect_tx(full, seg * nb);
+          for (int u = 0; u < nb; u++)
+            tma_bulk_g2s(smem_u32(s_slab + ((size_t)st * kB + u) * kSxRows), dval + (long long)(d0 + u) * P + rbase,
+                         seg, full);
+        }
+      }
+    }
+    return;
+  }
+  // consumers
+  const int nws = s_nw, tot = s_tot;
+  const bool all_staged = s_all;
+  auto stage_x = [&](long long b, int buf) {
+    const long long rb = b * kSxRows;
+    int w = 0;
+    for (int e = t * kE; e < tot; e += kTConsumers * kE) {
+      while (w + 1 < nws && e >= s_wsb[w + 1]) w++;
+      const long long g = rb + (s_wlo[w] & ~3) + (e - s_wsb[w]);
+      const long long avail = g < 0 ? 0 : (n - g) * (long long)sizeof(T);
+      const int bytes = avail <= 0 ? 0 : (avail >= 16 ? 16 : (int)avail);
+      cp_async16(s_xbuf + (size_t)buf * kCap + e, bytes ? (const void*)(x + g) : (const void*)x, bytes);
+    }
+    cp_async_commit();
+  };
+  if ((long long)blockIdx.x < nblk) stage_x(blockIdx.x, 0);
+  long long i = 0;
+  int it = 0;
+  for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x, it ^= 1) {
+    const long long rbase = blk * kSxRows;
+    if (blk + gridDim.x < nblk) stage_x(blk + gridDim.x, it ^ 1);
+    else cp_async_commit();
+    cp_async_wait<1>();
+    consumers_sync();  // this block's x windows have landed (every consumer's copies)
+    const T* sx = s_xbuf + (size_t)it * kCap;
+    acc_t acc[4] = {0, 0, 0, 0};
+    for (int b = 0; b < nbatch; b++, i++) {
+      const int st = (int)(i % kTStages);
+      mbar_wait(smem_u32(&s_full[st]), (unsigned)((i / kTStages) & 1));
+      const int d0 = b * kB, nb = nd - d0 < kB ? nd - d0 : kB;
+      const T* sl = s_slab + (size_t)st * kB * kSxRows + t;
+      if (nb == kB && all_staged) {  // fast path: unrolled, every x read from shared memory
+        if constexpr (sizeof(T) == 4 && kFp32Arith) {
+          float sq[4];
+#pragma unroll
+          for (int u = 0; u < kB; u++) {
+            const T* xs = sx + s_xb[d0 + u] + t;
+#pragma unroll
+            for (int q = 0; q < 4; q++)
+              sq[q] = u == 0 ? __fmul_rn(sl[q * kDiaThreads], xs[q * kDiaThreads])
+                             : __fmaf_rn(sl[u * kSxRows + q * kDiaThreads], xs[q * kDiaThreads], sq[q]);
+          }
+#pragma unroll
+          for (int q = 0; q < 4; q++) acc[q] += (acc_t)sq[q];
+        } else {
+#pragma unroll
+          for (int u = 0; u < kB; u++) {
+            const T* xs = sx + s_xb[d0 + u] + t;
+#pragma unroll
+            for (int q = 0; q < 4; q++) acc[q] += mulp(sl[u * kSxRows + q * kDiaThreads], xs[q * kDiaThreads]);
+          }
+        }
+      } else {
+        for (int u = 0; u < nb; u++) {
+          const int xb = s_xb[d0 + u], o = s_off[d0 + u];
+#pragma unroll
+          for (int q = 0; q < 4; q++) {
+            const long long c = rbase + t + q * kDiaThreads + o;
+            const T xv = xb >= 0 ? sx[xb + t + q * kDiaThreads] : (c >= 0 && c < n ? ld_x(x + c) : T(0));
+            acc[q] += mulp(sl[u * kSxRows + q * kDiaThreads], xv);
+          }
+        }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(smem_u32(&s_empty[st]));
+    }
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      const long long r = rbase + t + q * kDiaThreads;
+      if (r < m) y[r] = (T)acc[q];
+    }
+    consumers_sync();  // x buffer `it` is restaged in the next iteration
+  }
+  cp_async_wait<0>();
+  pdl_trigger();
+}
+
 struct MergeWork {
   int2* coords;
   int* crow;
@@ -1497,6 +1765,29 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
   const int* offs = (const int*)A->ptr[0];
   const T* dv = (const T*)A->ptr[1];
   const int nd = (int)A->ndiag;
+  if constexpr (!PUSH) {
+    // the TMA kernel for matrices of >= SFS_DIA_SX_MIN blocks of kSxRows rows (< 0: never).  Corpus-200
+    // DIA race (race_probe, us/rep): never 874, >= 296 blocks 816, 148: 802, 64: 800, 16: 820
+    static const long long sx_min = [] {
+      const char* e = getenv("SFS_DIA_SX_MIN");
+      return e ? atoll(e) : 64LL;
+    }();
+    const long long nsx = ceil_div(m, (long long)kSxRows);
+    if (sx_min >= 0 && nsx >= sx_min && nd >= 1 && nd <= kDiaSmemOffs && ((uintptr_t)x % 16) == 0) {
+      // TMA-streamed slab: 8 consumer warps + 1 producer warp per CTA
+      static std::once_flag attr_once[kMaxDevices];
+      int dev = 0;
+      if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+      std::call_once(attr_once[dev], [] {
+        cudaFuncSetAttribute(k_spmv_dia_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dia_tma_smem<T>());
+      });
+      constexpr int per_sm = (int)((228 * 1024) / (dia_tma_smem<T>() + 10 * 1024)) < 1
+                                 ? 1 : (int)((228 * 1024) / (dia_tma_smem<T>() + 10 * 1024));  // smem-bound
+      const int gt = (int)(nsx < (long long)kSMs * per_sm ? nsx : (long long)kSMs * per_sm);
+      return launch_k_smem(k_spmv_dia_tma<T>, dim3(gt), dim3(kTThreadsAll), dia_tma_smem<T>(), s, offs, dv, x, y, m,
+                           A->n, A->pitch, nd);
+    }
+  }
   if (dia_v4_enabled(sizeof(T))) {
     // L2 prefetch of the next batch's slab (SFS_DIA_PF: distance in batches, 0 = off; A/B switch).
     // 128^3 fp32 stencil cold (tools/ab_dia_pf.sh): off 54.3 us (0.69), 1: 52.2 us (0.71), 2: 53.2, 3: 55.3
