@@ -350,6 +350,7 @@ static sfs_status convert_impl(const DevCSR& d, sfs_format fmt, const sfs_featur
   A->pitch = pitch_of(d.m);
   A->stream = s;
   A->variant = f.csr_variant;
+  A->banded = (f.admissible_mask >> SFS_DIA) & 1u;
   A->user_free = g_user_free;  // the allocator this handle's buffers come from
   const size_t sv = vbytes(d.dtype);
   auto own = [&](size_t b) -> void* {

@@ -136,6 +136,8 @@ struct Matrix {
   int variant = 0;             // CSR: 0 vector, 1 merge, 2 stream, 3 tile, 4 tile + row-start bitmap,
                                // 5 tile + bitmap over the non-empty rows + row map;
                                // HYB: 1 = one launch (ptr[5] = ovf)
+  bool banded = false;         // DIA-admissible pattern (columns near the diagonal): the TMA ELL kernel
+                               // streams its slots while x reads hit L1 (gather-bound patterns keep LDG)
   void* work = nullptr;        // CSR merge / tile partition and carries
   cudaStream_t stream = nullptr;
   void (*user_free)(void*, void*) = nullptr;  // allocator hook at creation (nullptr: the library's pool)

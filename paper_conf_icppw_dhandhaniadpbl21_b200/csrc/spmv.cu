@@ -1650,6 +1650,132 @@ __global__ void __launch_bounds__(kTThreadsAll, 1) k_spmv_dia_tma(const int* __r
   pdl_trigger();
 }
 
+// ELL (and HYB without a COO part) for large banded matrices: the slot slabs (ecol, eval: slot-major,
+// contiguous per slot) streamed by TMA bulk copies through an mbarrier ring, as k_spmv_dia_tma; the
+// consumers read the column indices and values of their rows (t + 256 q) from shared memory
+// (conflict-free) and gather x through L1.  Measured (profiles/r02/micro_ab.txt): banded / block-diagonal /
+// stencil ELL 0.80-0.94 -> 0.90-0.96 of HBM cold; gather-bound (uniform) patterns and the HYB launch
+// shapes with an overflow walk got slower, so they keep k_spmv_ell.
+#ifndef SFS_ELL_TMA_KB
+#define SFS_ELL_TMA_KB 4  // slots per stage
+#endif
+#ifndef SFS_ELL_TMA_STAGES
+#define SFS_ELL_TMA_STAGES 3
+#endif
+template <typename T> constexpr size_t ell_tma_stage_bytes() { return (size_t)SFS_ELL_TMA_KB * kSxRows * (4 + sizeof(T)); }
+template <typename T> constexpr size_t ell_tma_smem() { return (size_t)SFS_ELL_TMA_STAGES * ell_tma_stage_bytes<T>(); }
+
+template <typename T>
+__global__ void __launch_bounds__(kTThreadsAll, 1) k_spmv_ell_tma(const int* __restrict__ ecol, const T* __restrict__ eval,
+                                                                  const T* __restrict__ x, T* __restrict__ y,
+                                                                  long long m, long long P, int K) {
+  constexpr int kB = SFS_ELL_TMA_KB;
+  constexpr int kStages = SFS_ELL_TMA_STAGES;
+  extern __shared__ __align__(128) unsigned char s_dyn[];
+  __shared__ __align__(8) unsigned long long s_full[kStages], s_empty[kStages];
+  const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+  if (t == 0) {
+    for (int i = 0; i < kStages; i++) {
+      mbar_init(smem_u32(&s_full[i]), 1);
+      mbar_init(smem_u32(&s_empty[i]), kTConsumers / 32);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  pdl_wait();
+  __syncthreads();
+  const long long nblk = ceil_div(m, (long long)kSxRows);
+  const int nbatch = (K + kB - 1) / kB;
+  // stage st: [kB][kSxRows] column indices, then [kB][kSxRows] values
+  auto scol = [&](int st) { return reinterpret_cast<int*>(s_dyn + (size_t)st * ell_tma_stage_bytes<T>()); };
+  auto sval = [&](int st) {
+    return reinterpret_cast<T*>(s_dyn + (size_t)st * ell_tma_stage_bytes<T>() + (size_t)kB * kSxRows * 4);
+  };
+  if (warp == kTConsumers / 32) {  // producer warp
+    if (lane == 0) {
+      long long i = 0;
+      for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+        const long long rbase = blk * kSxRows;
+        const long long rows = P - rbase < kSxRows ? P - rbase : kSxRows;  // P: multiple of 32, >= m
+        for (int b = 0; b < nbatch; b++, i++) {
+          const int st = (int)(i % kStages);
+          const long long round = i / kStages;
+          if (round > 0) mbar_wait(smem_u32(&s_empty[st]), (unsigned)((round - 1) & 1));
+          const int j0 = b * kB, nb = K - j0 < kB ? K - j0 : kB;
+          const unsigned full = smem_u32(&s_full[st]);
+          mbar_expect_tx(full, (unsigned)(rows * (4 + (long long)sizeof(T)) * nb));
+          for (int u = 0; u < nb; u++) {
+            tma_bulk_g2s(smem_u32(scol(st) + (size_t)u * kSxRows), ecol + (long long)(j0 + u) * P + rbase,
+                         (unsigned)(rows * 4), full);
+            tma_bulk_g2s(smem_u32(sval(st) + (size_t)u * kSxRows), eval + (long long)(j0 + u) * P + rbase,
+                         (unsigned)(rows * (long long)sizeof(T)), full);
+          }
+        }
+      }
+    }
+    return;
+  }
+  long long i = 0;
+  for (long long blk = blockIdx.x; blk < nblk; blk += gridDim.x) {
+    const long long rbase = blk * kSxRows;
+    const bool full = rbase + kSxRows <= m;
+    acc_t acc[4] = {0, 0, 0, 0};
+    for (int b = 0; b < nbatch; b++, i++) {
+      const int st = (int)(i % kStages);
+      mbar_wait(smem_u32(&s_full[st]), (unsigned)((i / kStages) & 1));
+      const int j0 = b * kB, nb = K - j0 < kB ? K - j0 : kB;
+      const int* sc = scol(st) + t;
+      const T* sv = sval(st) + t;
+      if (nb == kB && full) {
+        int c[kB][4];
+        T v[kB][4], xv[kB][4];
+#pragma unroll
+        for (int u = 0; u < kB; u++)
+#pragma unroll
+          for (int q = 0; q < 4; q++) {
+            c[u][q] = sc[u * kSxRows + q * kDiaThreads];
+            v[u][q] = sv[u * kSxRows + q * kDiaThreads];
+          }
+#pragma unroll
+        for (int u = 0; u < kB; u++)
+#pragma unroll
+          for (int q = 0; q < 4; q++) xv[u][q] = c[u][q] >= 0 ? ld_x(x + c[u][q]) : T(0);  // padding: (-1, +0)
+        if constexpr (sizeof(T) == 4 && kFp32Arith) {
+          float sq[4];
+#pragma unroll
+          for (int q = 0; q < 4; q++) {
+            sq[q] = __fmul_rn(v[0][q], xv[0][q]);
+#pragma unroll
+            for (int u = 1; u < kB; u++) sq[q] = __fmaf_rn(v[u][q], xv[u][q], sq[q]);
+            acc[q] += (acc_t)sq[q];
+          }
+        } else {
+#pragma unroll
+          for (int u = 0; u < kB; u++)
+#pragma unroll
+            for (int q = 0; q < 4; q++) acc[q] += mulp(v[u][q], xv[u][q]);
+        }
+      } else {
+        // rows past the copied segment (the last block's rows >= P) hold stale shared memory: rows >= m
+        // are skipped
+        for (int u = 0; u < nb; u++)
+#pragma unroll
+          for (int q = 0; q < 4; q++) {
+            const int c = rbase + t + q * kDiaThreads < m ? sc[u * kSxRows + q * kDiaThreads] : -1;
+            if (c >= 0) acc[q] += mulp(sv[u * kSxRows + q * kDiaThreads], ld_x(x + c));
+          }
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(smem_u32(&s_empty[st]));
+    }
+#pragma unroll
+    for (int q = 0; q < 4; q++) {
+      const long long r = rbase + t + q * kDiaThreads;
+      if (r < m) y[r] = (T)acc[q];
+    }
+  }
+  pdl_trigger();
+}
+
 struct MergeWork {
   int2* coords;
   int* crow;
@@ -1705,6 +1831,31 @@ cudaError_t launch_zero(T* y, long long m, cudaStream_t s) {
 template <typename T, bool PUSH = false, bool ATOM = false>
 cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s, int early_trigger,
                        PushParam<PUSH> push = {}) {
+  if constexpr (!PUSH) {
+    // the TMA kernel for slabs of >= SFS_ELL_TMA_MB megabytes (default 256 = 2 x L2; < 0: never).  In the
+    // race's back-to-back reps an L2-resident ELL keeps k_spmv_ell: gating on >= 64 row blocks instead made
+    // the corpus-200 ELL race 5 % slower (mid-size bands with few slots: 1.2-3.6x per matrix)
+    static const long long tma_mb = [] {
+      const char* e = getenv("SFS_ELL_TMA_MB");
+      return e ? atoll(e) : 256LL;
+    }();
+    const long long nb = ceil_div(A->m, (long long)kSxRows);
+    const long long slab = (long long)K * A->pitch * (4 + (long long)sizeof(T));
+    if (!ATOM && tma_mb >= 0 && slab >= tma_mb * (1ll << 20) && K >= 1 && A->banded &&
+        (A->fmt == SFS_ELL || A->coo_nnz == 0)) {
+      static std::once_flag attr_once[kMaxDevices];
+      int dev = 0;
+      if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= kMaxDevices) return cudaErrorInvalidDevice;
+      std::call_once(attr_once[dev], [] {
+        cudaFuncSetAttribute(k_spmv_ell_tma<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ell_tma_smem<T>());
+      });
+      constexpr int per_sm = (int)((228 * 1024) / (ell_tma_smem<T>() + 2 * 1024)) < 1
+                                 ? 1 : (int)((228 * 1024) / (ell_tma_smem<T>() + 2 * 1024));
+      const int gt = (int)(nb < (long long)kSMs * per_sm ? nb : (long long)kSMs * per_sm);
+      return launch_k_smem(k_spmv_ell_tma<T>, dim3(gt), dim3(kTThreadsAll), ell_tma_smem<T>(), s,
+                           (const int*)A->ptr[0], (const T*)A->ptr[1], x, y, A->m, A->pitch, K);
+    }
+  }
   const long long groups = A->pitch / 4;
   const int S = split_factor(groups, K, 2 * ell_batch<T>(), 16);
   const long long niter = ceil_div(groups, kEllThreads / S);
