@@ -1027,6 +1027,9 @@ constexpr long long kHybRowwiseLarge = 32;
 
 // ATOM (HYB with long overflow rows, overlapped): y was zeroed ahead and the COO part runs concurrently,
 // so the ELL part adds its row sums atomically instead of storing them.
+#ifndef SFS_OVF_BATCH
+#define SFS_OVF_BATCH 2  // HYB overflow entries per walk step (corpus HYB race: 1: 2683, 2: 2668, 3: 2677, 4: 2687, 8: 2757 us/rep)
+#endif
 template <typename T, bool OVF, bool PUSH = false, bool ATOM = false>
 __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const int* __restrict__ ecol,
                                                                          const T* __restrict__ eval,
@@ -1102,13 +1105,14 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
         if (c.w >= 0) acc[3] += mulp(v.v[3], ld_x(x + c.w));
       }
       if (OVF) {
-        // the 4 rows' overflow entries are contiguous: [ob[0], ob[4]); batches of 4 (clamped loads),
+        // the 4 rows' overflow entries are contiguous: [ob[0], ob[4]); batches of kOB (clamped loads),
         // batch b taken by slot-part b mod S, so the parts share the walk
-        for (int k = ob[0] + 4 * p; k < ob[4]; k += 4 * S) {
-          int c[4];
-          T v[4];
+        constexpr int kOB = SFS_OVF_BATCH;
+        for (int k = ob[0] + kOB * p; k < ob[4]; k += kOB * S) {
+          int c[kOB];
+          T v[kOB];
 #pragma unroll
-          for (int u = 0; u < 4; u++) {
+          for (int u = 0; u < kOB; u++) {
             const int kk = k + u < ob[4] ? k + u : ob[4] - 1;
 #ifdef SFS_OVF_STREAM
             c[u] = ld_stream(ocol + kk);
@@ -1121,7 +1125,7 @@ __global__ void __launch_bounds__(kEllThreads, ell_ctas<T>()) k_spmv_ell(const i
 #endif
           }
 #pragma unroll
-          for (int u = 0; u < 4; u++) {
+          for (int u = 0; u < kOB; u++) {
             const acc_t t = mulp(v[u], ld_x(x + c[u]));
             const int kk = k + u;
             if (kk < ob[4]) {
