@@ -84,7 +84,7 @@ def run_all():
             check_spmv(A, sfs.DIA, M, sfsgen.vector(seed, A.n, A.dtype), A.dtype, ctx=f"dia_sx {name}")
         M.free()
         n_ok += 1
-    print(f"DIA_SX_OK {n_ok}")
+    print(f"DIA_TMA_OK {n_ok}")
 
 
 def test_dia_tma_every_size():
@@ -92,4 +92,4 @@ def test_dia_tma_every_size():
     code = f"import sys; sys.path.insert(0, {HERE!r}); import test_gpu_dia_tma as t; t.run_all()"
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=240,
                        cwd=os.path.dirname(HERE))
-    assert r.returncode == 0 and f"DIA_SX_OK {len(cases())}" in r.stdout, r.stdout[-3000:] + r.stderr[-3000:]
+    assert r.returncode == 0 and f"DIA_TMA_OK {len(cases())}" in r.stdout, r.stdout[-3000:] + r.stderr[-3000:]
