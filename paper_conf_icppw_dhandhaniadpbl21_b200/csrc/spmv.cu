@@ -602,6 +602,9 @@ __global__ void k_spmv_csr_merge_fixup(const int* __restrict__ carry_row, const 
 // the first chunk's loads and x gathers overlap it; the kernel waits before touching y.  No full zero
 // pass, no row array: CSR's own bytes only.
 constexpr int kTThreads = 256;
+#ifndef SFS_TILE_PFD
+#define SFS_TILE_PFD 1  // chunks ahead of the L2 prefetch of col / val (A/B builds)
+#endif
 #ifndef SFS_TILE_CTAS
 #define SFS_TILE_CTAS 4  // CTAs per SM of the tile kernel (register cap; A/B builds set 5)
 #endif
@@ -681,9 +684,9 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     const long long k = k0 + l * kTV;
     // footprints >> L2 (pf): the next chunk's col (1 KB) and val (1 / 2 KB) into L2, one 128-byte line
     // per lane (L2-resident matrices skip it: there the prefetches only cost issue slots)
-    if (pf && ch + 1 < ce) {
+    if (pf && ch + SFS_TILE_PFD < ce) {
       constexpr int kColLines = kTChunk * 4 / 128;
-      const long long kn = k0 + kTChunk;
+      const long long kn = k0 + (long long)SFS_TILE_PFD * kTChunk;
       const long long e = l < kColLines ? kn + l * 32 : kn + (long long)(l - kColLines) * (128 / (long long)sizeof(T));
       if (l < kColLines + kTChunk * (int)sizeof(T) / 128 && e < z) {
         const void* a = l < kColLines ? (const void*)(col + e) : (const void*)(val + e);
