@@ -1528,6 +1528,7 @@ __global__ void __launch_bounds__(kTThreadsAll, 1) k_spmv_dia_tma(const int* __r
                                                                   long long m, long long n, long long P, int nd) {
   constexpr int kB = dia_tma_batch<T>();
   constexpr int kTStages = dia_tma_stages<T>();
+  static_assert(kTStages >= 1 && kTStages <= 16, "the mbarrier arrays hold 16 stages");
   constexpr int kCap = dia_tma_xbuf<T>() / (int)sizeof(T);
   constexpr int kE = 16 / (int)sizeof(T);
   extern __shared__ __align__(128) unsigned char s_dyn[];
