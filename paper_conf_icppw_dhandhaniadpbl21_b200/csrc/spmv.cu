@@ -658,7 +658,8 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
                                               const T* __restrict__ val, const T* __restrict__ x, T* __restrict__ y,
                                               long long m, long long z, long long cpw, long long warp,
                                               const int* __restrict__ ca, const int* __restrict__ srow,
-                                              long long nwarps, int* head, const unsigned* __restrict__ bm, int pf,
+                                              long long nwarps, int* head, const unsigned* __restrict__ bm,
+                                              const unsigned short* __restrict__ pb, int pf,
                                               const int* __restrict__ ne) {
   const int l = threadIdx.x & 31;
   const long long nchunks = ceil_div(z, kTChunk);
@@ -694,8 +695,18 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
       }
     }
     const int a_lo = BM ? 0 : __ldg(ca + ch), a_hi = BM ? 0 : __ldg(ca + ch + 1);
+    // variant 4 reads its lane's bitmap byte with the row starts of the chunk's earlier bytes (k_tile_pack);
+    // variant 5 scans the bitmap bytes (corpus CSR race -1.3 % with the packed form, R-MAT 2^22 +5 %)
+    constexpr bool kPack = BM && !MAP;
     unsigned sb = 0;
-    if (BM) sb = (__ldg(bm + ch * (kTChunk / 32) + (l >> 2)) >> ((l & 3) * 8)) & 0xFFu;
+    int spre = 0;  // row starts in the chunk before this lane's entries
+    if (kPack) {
+      const unsigned pv = __ldg(pb + ch * 32 + l);
+      sb = pv & 0xFFu;
+      spre = (int)(pv >> 8);
+    } else if (BM) {
+      sb = (__ldg(bm + ch * (kTChunk / 32) + (l >> 2)) >> ((l & 3) * 8)) & 0xFFu;
+    }
     acc_t p[kTV];
     {
       int c[kTV];
@@ -724,17 +735,20 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     }
     int r[kTV];
     if (BM) {
-      const int cnt = __popc(sb);
-      int inc = cnt;
+      if (!kPack) {  // exclusive warp scan of the bytes' popcounts
+        const int cnt = __popc(sb);
+        int inc = cnt;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const int u = __shfl_up_sync(0xffffffffu, inc, o);
-        if (l >= o) inc += u;
+        for (int o = 1; o < 32; o <<= 1) {
+          const int u = __shfl_up_sync(0xffffffffu, inc, o);
+          if (l >= o) inc += u;
+        }
+        spre = inc - cnt;
       }
-      const int base = a_run - 1 + inc - cnt;
+      const int base = a_run - 1 + spre;
 #pragma unroll
       for (int i = 0; i < kTV; i++) r[i] = base + __popc(sb & ((2u << i) - 1u));
-      a_run += __shfl_sync(0xffffffffu, inc, 31);
+      a_run += __shfl_sync(0xffffffffu, spre + __popc(sb), 31);
     } else {
     // start marks of the rows beginning in this chunk (non-empty rows start at distinct positions)
     reinterpret_cast<int4*>(head)[2 * l] = make_int4(-1, -1, -1, -1);
@@ -829,13 +843,14 @@ __global__ void __launch_bounds__(kTThreads, SFS_TILE_CTAS) k_spmv_csr_tile(cons
                                                                T* __restrict__ y, long long m, long long z,
                                                                long long cpw, long long nwarps,
                                                                const int* __restrict__ ca, const int* __restrict__ srow,
-                                                               const unsigned* __restrict__ bm, int pf,
+                                                               const unsigned* __restrict__ bm,
+                                                               const unsigned short* __restrict__ pb, int pf,
                                                                const int* __restrict__ ne) {
   __shared__ __align__(16) int s_head[BM ? 1 : kTThreads / 32][kTChunk];
   const long long warp = ((long long)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   if (warp < nwarps)
     csr_tile_warp<T, VEC, BM, MAP>(rp, col, val, x, y, m, z, cpw, warp, ca, srow, nwarps,
-                                   s_head[BM ? 0 : threadIdx.x >> 5], bm, pf, ne);
+                                   s_head[BM ? 0 : threadIdx.x >> 5], bm, pb, pf, ne);
   else
     pdl_wait();
   pdl_trigger();
@@ -878,6 +893,22 @@ __global__ void k_row_starts(const int* __restrict__ rp, long long m, unsigned* 
     if (__ldg(rp + r + 1) > k) {
       atomicOr(bm + (k >> 5), 1u << (k & 31));
       if (ne) ne[pos[r]] = (int)r;
+    }
+  }
+}
+
+// per chunk and lane: (row starts in the chunk's bytes before the lane's) << 8 | the lane's bitmap byte (<= 248
+// starts precede lane 31), so the tile kernel reads its row offsets instead of scanning the bitmap bytes
+__global__ void k_tile_pack(const unsigned* __restrict__ bm, long long nchunks, unsigned short* __restrict__ pb) {
+  for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nchunks; c += (long long)gridDim.x * blockDim.x) {
+    unsigned run = 0;
+    for (int w = 0; w < kTChunk / 32; w++) {
+      const unsigned word = bm[c * (kTChunk / 32) + w];
+      for (int b = 0; b < 4; b++) {
+        const unsigned byte = (word >> (8 * b)) & 0xFFu;
+        pb[c * 32 + w * 4 + b] = (unsigned short)((run << 8) | byte);
+        run += __popc(byte);
+      }
     }
   }
 }
@@ -1805,6 +1836,7 @@ struct TileWork {
   int* a;        // a_c = lower_bound(rp, 256 c), c = 0..nchunks
   int* srow;     // row split at the start of each warp range (m: none)
   unsigned* bm;  // variants 4, 5: row-start bitmap, nchunks * 8 words
+  unsigned short* pb;  // variants 4, 5: per chunk and lane, (row starts in the chunk's earlier bytes << 8) | byte
   int* ne;       // variant 5: row of each non-empty-row rank (m entries reserved)
 };
 TileWork tile_work(void* base, const TileGeom& g) {
@@ -1816,6 +1848,8 @@ TileWork tile_work(void* base, const TileGeom& g) {
   p += al256(sizeof(int) * g.nwarps);
   w.bm = (unsigned*)p;
   p += al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32));
+  w.pb = (unsigned short*)p;
+  p += al256(sizeof(unsigned short) * g.nchunks * 32);
   w.ne = (int*)p;
   return w;
 }
@@ -2031,7 +2065,7 @@ cudaError_t spmv_t(const Matrix* A, const T* x, T* y, cudaStream_t s) {
         const int pf = pf_mb >= 0 && foot > pf_mb * (1ll << 20);
         auto go = [&](auto kern) {
           return launch_k(kern, grid, dim3(tpb), s, rp, col, val, x, y, m, z, g.cpw, g.nwarps, (const int*)w.a,
-                          (const int*)w.srow, (const unsigned*)w.bm, pf, (const int*)w.ne);
+                          (const int*)w.srow, (const unsigned*)w.bm, (const unsigned short*)w.pb, pf, (const int*)w.ne);
         };
         if (A->variant == 5) {  // empty rows: all of y zeroed ahead (PDL-overlapped), ranks mapped to rows
           e = launch_zero<T>(y, m, s);
@@ -2151,7 +2185,7 @@ cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, vo
 size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
   const TileGeom g = tile_geom(z);
   return al256(sizeof(int) * (g.nchunks + 1)) + al256(sizeof(int) * g.nwarps) +
-         (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) : 0) +
+         (bitmap ? al256(sizeof(unsigned) * g.nchunks * (kTChunk / 32)) + al256(sizeof(unsigned short) * g.nchunks * 32) : 0) +
          (bitmap == 2 ? al256(sizeof(int) * m) : 0);
 }
 
@@ -2180,6 +2214,8 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
       if (e != cudaSuccess) return e;
     }
     k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
+    count_launch();
+    k_tile_pack<<<grid_cap(g.nchunks, 256, 8), 256, 0, s>>>(w.bm, g.nchunks, w.pb);
     count_launch();
     if (bitmap == 2) {
       const long long items = std::max(g.nchunks + 1, g.nwarps);
