@@ -623,23 +623,15 @@ TileGeom tile_geom(long long z) {
   return g;
 }
 
+// a[c] = lower_bound(rp, 256 c) (c < nchunks), a[nchunks] = m: one pass over the rows instead of a binary search
+// per chunk (a row r owns the chunk starts in (rp[r-1], rp[r]], row 0 the start 0)
 __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, long long nchunks, int* __restrict__ a) {
-  for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c <= nchunks;
-       c += (long long)gridDim.x * blockDim.x) {
-    long long v;
-    if (c == 0) v = 0;
-    else if (c == nchunks) v = m;
-    else {
-      const long long k = c * kTChunk;
-      long long lo = 0, hi = m;  // first row r with rp[r] >= k
-      while (lo < hi) {
-        const long long mid = (lo + hi) >> 1;
-        if (rp[mid] < k) lo = mid + 1;
-        else hi = mid;
-      }
-      v = lo;
-    }
-    a[c] = (int)v;
+  for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r <= m; r += (long long)gridDim.x * blockDim.x) {
+    const long long hi = __ldg(rp + r);
+    long long c = r == 0 ? 0 : __ldg(rp + r - 1) / kTChunk + 1;
+    const long long ce = hi / kTChunk < nchunks - 1 ? hi / kTChunk : nchunks - 1;
+    for (; c <= ce; c++) a[c] = (int)r;
+    if (r == m) a[nchunks] = (int)m;
   }
 }
 
@@ -869,18 +861,15 @@ __global__ void k_zero_rows(T* __restrict__ y, const int* __restrict__ srow, lon
   }
 }
 
-// srow[w] = the row holding the first entry of warp w's range if it started before it, else m
-__global__ void k_tile_split_rows(const int* __restrict__ rp, long long m, long long cpw, long long nwarps,
-                                  int* __restrict__ srow) {
+// srow[w] = the row holding the first entry of warp w's range if it started before it, else m; from the
+// chunk partition: with r0 = a[w cpw] (the first row with rp[r0] >= kb), the entry kb starts row r0 iff
+// rp[r0] == kb, else it lies inside row r0 - 1
+__global__ void k_tile_split_rows(const int* __restrict__ rp, const int* __restrict__ a, long long m, long long cpw,
+                                  long long nwarps, int* __restrict__ srow) {
   for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nwarps; w += (long long)gridDim.x * blockDim.x) {
     const long long kb = w * cpw * kTChunk;
-    long long lo = 0, hi = m;  // last row r with rp[r] <= kb
-    while (lo < hi) {
-      const long long mid = (lo + hi + 1) >> 1;
-      if (rp[mid] <= kb) lo = mid;
-      else hi = mid - 1;
-    }
-    srow[w] = (w > 0 && rp[lo] < kb) ? (int)lo : (int)m;
+    const int r0 = __ldg(a + w * cpw);
+    srow[w] = (w > 0 && (long long)__ldg(rp + r0) != kb) ? r0 - 1 : (int)m;
   }
 }
 
@@ -2192,9 +2181,9 @@ size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
   const TileGeom g = tile_geom(z);
   TileWork w = tile_work(work, g);
-  k_csr_tile_partition<<<grid_cap(g.nchunks + 1, 256, 8), 256, 0, s>>>(rp, m, g.nchunks, w.a);
+  k_csr_tile_partition<<<grid_cap(m + 1, 256, 8), 256, 0, s>>>(rp, m, g.nchunks, w.a);
   count_launch();
-  k_tile_split_rows<<<grid_cap(g.nwarps, 256, 8), 256, 0, s>>>(rp, m, g.cpw, g.nwarps, w.srow);
+  k_tile_split_rows<<<grid_cap(g.nwarps, 256, 8), 256, 0, s>>>(rp, w.a, m, g.cpw, g.nwarps, w.srow);
   count_launch();
   if (bitmap) {
     cudaError_t e = cudaMemsetAsync(w.bm, 0, sizeof(unsigned) * g.nchunks * (kTChunk / 32), s);
