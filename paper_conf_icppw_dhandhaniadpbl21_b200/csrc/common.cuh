@@ -2,10 +2,39 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include "shape.h"
 
 namespace sfs {
+
+// ---------------------------------------------------------------- programmatic dependent launch
+// The feature, conversion and preparation chains run as PDL chains like the SpMV kernels: every kernel
+// waits (griddepcontrol.wait: a no-op without a programmatic predecessor) before touching memory and
+// releases its successor when its work is done; launch_dep sets the launch attribute (SFS_PDL=0: off).
+__device__ __forceinline__ void dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void dep_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+inline bool dep_enabled() {
+  static const bool v = [] {
+    const char* e = getenv("SFS_PDL");
+    return !(e && e[0] == '0');
+  }();
+  return v;
+}
+template <typename... Params, typename... Args>
+cudaError_t launch_dep(void (*kern)(Params...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = s;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = dep_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<Params>(args)...);
+}
 
 
 // ---------------------------------------------------------------- cache-hinted loads

@@ -43,6 +43,7 @@ __global__ void __launch_bounds__(kTileThreads) k_csr2coo(const int* __restrict_
                                                           const T* __restrict__ val, long long m, long long z,
                                                           int* __restrict__ orow, int* __restrict__ ocol,
                                                           T* __restrict__ oval) {
+  dep_wait();
   __shared__ int s_rp[kTile + 2];
   __shared__ int s_row[kTile];
   __shared__ int s_coord[4];
@@ -67,6 +68,7 @@ __global__ void __launch_bounds__(kTileThreads) k_csr2coo(const int* __restrict_
     ocol[k0 + i] = col[k0 + i];
     oval[k0 + i] = val[k0 + i];
   }
+  dep_trigger();
 }
 
 // ELL slab (also the ELL part of HYB).  A CTA owns 128 consecutive rows; their CSR segment is
@@ -82,6 +84,7 @@ template <typename T>
 __global__ void __launch_bounds__(kEllRows) k_csr2ell(const int* __restrict__ rp, const int* __restrict__ col,
                                                       const T* __restrict__ val, long long m, long long P, int K,
                                                       int cap, int* __restrict__ ecol, T* __restrict__ eval) {
+  dep_wait();
   extern __shared__ __align__(16) unsigned char s_seg[];
   T* s_val = (T*)s_seg;                          // [cap]
   int* s_col = (int*)(s_seg + sizeof(T) * cap);  // [cap]
@@ -111,6 +114,7 @@ __global__ void __launch_bounds__(kEllRows) k_csr2ell(const int* __restrict__ rp
     ecol[(long long)j * P + r] = c;
     eval[(long long)j * P + r] = v;
   }
+  dep_trigger();
 }
 
 // COO part of HYB: entries j >= K of row r go to ovf[r] + (j - K).
@@ -119,6 +123,7 @@ __global__ void __launch_bounds__(kTileThreads) k_hyb_coo_part(const int* __rest
                                                                const T* __restrict__ val, long long m, long long z, int K,
                                                                const int* __restrict__ ovf, int* __restrict__ crow,
                                                                int* __restrict__ ccol, T* __restrict__ cval) {
+  dep_wait();
   __shared__ int s_rp[kTile + 2];
   __shared__ int s_coord[4];
   long long d0, d1;
@@ -141,10 +146,12 @@ __global__ void __launch_bounds__(kTileThreads) k_hyb_coo_part(const int* __rest
     }
     k++;
   }
+  dep_trigger();
 }
 
 __global__ void k_dia_offsets(const unsigned* __restrict__ bitmap, long long nw, const int* __restrict__ wprefix,
                               long long m, int* __restrict__ offs) {
+  dep_wait();
   for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nw; w += (long long)gridDim.x * blockDim.x) {
     unsigned b = bitmap[w];
     int o = wprefix[w];
@@ -154,6 +161,7 @@ __global__ void k_dia_offsets(const unsigned* __restrict__ bitmap, long long nw,
       b &= b - 1;
     }
   }
+  dep_trigger();
 }
 
 // DIA scatter: thread per row; the j-th entry of consecutive rows usually sits on the same diagonal,
@@ -162,6 +170,7 @@ template <typename T>
 __global__ void k_csr2dia(const int* __restrict__ rp, const int* __restrict__ col, const T* __restrict__ val,
                           long long m, long long P, const unsigned* __restrict__ bitmap,
                           const int* __restrict__ wprefix, T* __restrict__ dval) {
+  dep_wait();
   for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (long long)gridDim.x * blockDim.x) {
     const int b = rp[r], e = rp[r + 1];
     for (int k = b; k < e; k++) {
@@ -172,6 +181,7 @@ __global__ void k_csr2dia(const int* __restrict__ rp, const int* __restrict__ co
       dval[d * P + r] = val[k];
     }
   }
+  dep_trigger();
 }
 
 int grid_cap(long long items, int threads, int per_sm) {
@@ -186,9 +196,9 @@ cudaError_t launch_csr2coo(int dtype, const int* rp, const int* col, const void*
   long long tiles = ceil_div(m + z, kTile);
   if (z == 0) return cudaSuccess;
   if (dtype == SFS_F64)
-    k_csr2coo<double><<<(unsigned)tiles, kTileThreads, 0, s>>>(rp, col, (const double*)val, m, z, orow, ocol, (double*)oval);
+    (void)launch_dep(k_csr2coo<double>, dim3((unsigned)tiles), dim3(kTileThreads), 0, s, rp, col, (const double*)val, m, z, orow, ocol, (double*)oval);
   else
-    k_csr2coo<float><<<(unsigned)tiles, kTileThreads, 0, s>>>(rp, col, (const float*)val, m, z, orow, ocol, (float*)oval);
+    (void)launch_dep(k_csr2coo<float>, dim3((unsigned)tiles), dim3(kTileThreads), 0, s, rp, col, (const float*)val, m, z, orow, ocol, (float*)oval);
   count_launch();
   return cudaGetLastError();
 }
@@ -208,10 +218,10 @@ cudaError_t launch_csr2ell(int dtype, const int* rp, const int* col, const void*
     cudaFuncSetAttribute(k_csr2ell<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, kSegCapMax * 8);
   });
   if (dtype == SFS_F64)
-    k_csr2ell<double><<<g, kEllRows, cap * 12, s>>>(rp, col, (const double*)val, m, P, K, (int)cap, ecol,
+    (void)launch_dep(k_csr2ell<double>, dim3(g), dim3(kEllRows), cap * 12, s, rp, col, (const double*)val, m, P, K, (int)cap, ecol,
                                                     (double*)eval);
   else
-    k_csr2ell<float><<<g, kEllRows, cap * 8, s>>>(rp, col, (const float*)val, m, P, K, (int)cap, ecol,
+    (void)launch_dep(k_csr2ell<float>, dim3(g), dim3(kEllRows), cap * 8, s, rp, col, (const float*)val, m, P, K, (int)cap, ecol,
                                                   (float*)eval);
   count_launch();
   return cudaGetLastError();
@@ -222,10 +232,10 @@ cudaError_t launch_hyb_coo_part(int dtype, const int* rp, const int* col, const 
   if (z == 0) return cudaSuccess;
   long long tiles = ceil_div(m + z, kTile);
   if (dtype == SFS_F64)
-    k_hyb_coo_part<double><<<(unsigned)tiles, kTileThreads, 0, s>>>(rp, col, (const double*)val, m, z, K, ovf, crow,
+    (void)launch_dep(k_hyb_coo_part<double>, dim3((unsigned)tiles), dim3(kTileThreads), 0, s, rp, col, (const double*)val, m, z, K, ovf, crow,
                                                                      ccol, (double*)cval);
   else
-    k_hyb_coo_part<float><<<(unsigned)tiles, kTileThreads, 0, s>>>(rp, col, (const float*)val, m, z, K, ovf, crow,
+    (void)launch_dep(k_hyb_coo_part<float>, dim3((unsigned)tiles), dim3(kTileThreads), 0, s, rp, col, (const float*)val, m, z, K, ovf, crow,
                                                                     ccol, (float*)cval);
   count_launch();
   return cudaGetLastError();
@@ -233,7 +243,7 @@ cudaError_t launch_hyb_coo_part(int dtype, const int* rp, const int* col, const 
 
 cudaError_t launch_dia_offsets(const unsigned* bitmap, long long nw, const int* wprefix, long long m, int* offs,
                                cudaStream_t s) {
-  k_dia_offsets<<<grid_cap(nw, 256, 8), 256, 0, s>>>(bitmap, nw, wprefix, m, offs);
+  (void)launch_dep(k_dia_offsets, dim3(grid_cap(nw, 256, 8)), dim3(256), 0, s, bitmap, nw, wprefix, m, offs);
   count_launch();
   return cudaGetLastError();
 }
@@ -241,9 +251,9 @@ cudaError_t launch_dia_offsets(const unsigned* bitmap, long long nw, const int* 
 cudaError_t launch_csr2dia(int dtype, const int* rp, const int* col, const void* val, long long m, long long P,
                            const unsigned* bitmap, const int* wprefix, void* dval, cudaStream_t s) {
   if (dtype == SFS_F64)
-    k_csr2dia<double><<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, col, (const double*)val, m, P, bitmap, wprefix, (double*)dval);
+    (void)launch_dep(k_csr2dia<double>, dim3(grid_cap(m, 256, 8)), dim3(256), 0, s, rp, col, (const double*)val, m, P, bitmap, wprefix, (double*)dval);
   else
-    k_csr2dia<float><<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, col, (const float*)val, m, P, bitmap, wprefix, (float*)dval);
+    (void)launch_dep(k_csr2dia<float>, dim3(grid_cap(m, 256, 8)), dim3(256), 0, s, rp, col, (const float*)val, m, P, bitmap, wprefix, (float*)dval);
   count_launch();
   return cudaGetLastError();
 }

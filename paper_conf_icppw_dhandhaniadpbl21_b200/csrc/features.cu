@@ -37,6 +37,7 @@ __device__ __forceinline__ T warp_max(T v) {
 
 __global__ void __launch_bounds__(kRowThreads) k_rowstats(const int* __restrict__ rp, long long m, long long z,
                                                           DevAggr* __restrict__ ag, unsigned* __restrict__ hist) {
+  dep_wait();
   __shared__ unsigned sh_hist[kHistCap + 1];
   __shared__ unsigned long long sh_red[kRowThreads / 32][11];
   for (int i = threadIdx.x; i <= kHistCap; i += blockDim.x) sh_hist[i] = 0;
@@ -93,6 +94,7 @@ __global__ void __launch_bounds__(kRowThreads) k_rowstats(const int* __restrict_
   }
   for (int i = threadIdx.x; i <= kHistCap; i += blockDim.x)
     if (sh_hist[i]) atomicAdd(&hist[i], sh_hist[i]);
+  dep_trigger();
 }
 
 // merge-path tile over (row ends, nnz): column checks + diagonal bitmap
@@ -100,6 +102,7 @@ __global__ void __launch_bounds__(kNnzThreads) k_nnzpass(const int* __restrict__
                                                          long long m, long long n, long long z,
                                                          DevAggr* __restrict__ ag, unsigned* __restrict__ bitmap,
                                                          long long words) {
+  dep_wait();
   if (ag->flags & (FLAG_RP0 | FLAG_RP_DECREASE | FLAG_RP_END)) return;  // row_ptr invalid: do not walk it
   __shared__ int s_rp[kNnzTile + 2];
   __shared__ int s_col[kNnzTile];
@@ -159,14 +162,17 @@ __global__ void __launch_bounds__(kNnzThreads) k_nnzpass(const int* __restrict__
     long long gw = base / 32 + i;
     if (b && gw >= 0 && gw < words) atomicOr(&bitmap[gw], b);
   }
+  dep_trigger();
 }
 
 __global__ void k_popcount(const unsigned* __restrict__ bitmap, long long words, DevAggr* __restrict__ ag) {
+  dep_wait();
   unsigned long long c = 0;
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += (long long)gridDim.x * blockDim.x)
     c += __popc(bitmap[i]);
   c = warp_sum(c);
   if ((threadIdx.x & 31) == 0 && c) atomicAdd(&ag->ndiag, c);
+  dep_trigger();
 }
 
 // One CTA of kSelThreads.  j = rmax + 1.  The HYB width rule of Q6 (smallest k >= 1 with R(k) <= rmax,
@@ -183,6 +189,7 @@ __device__ __forceinline__ void publish(const DevAggr* ag, DevAggr* host_out) {
 __global__ void __launch_bounds__(kSelThreads) k_hyb_select(long long m, long long j, DevAggr* __restrict__ ag,
                                                             const unsigned* __restrict__ hist,
                                                             DevAggr* __restrict__ host_out) {
+  dep_wait();
   __shared__ long long s_w[kSelThreads / 32];
   __shared__ long long s_L;
   const int t = threadIdx.x, l = t & 31, w = t >> 5;
@@ -250,17 +257,21 @@ __global__ void __launch_bounds__(kSelThreads) k_hyb_select(long long m, long lo
       publish(ag, host_out);
     }
   }
+  dep_trigger();
 }
 
 __global__ void k_len_hist_range(const int* __restrict__ rp, long long m, long long lo, long long hi, long long wdt,
                                  unsigned* __restrict__ hist) {
+  dep_wait();
   for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (long long)gridDim.x * blockDim.x) {
     long long len = (long long)rp[r + 1] - rp[r];
     if (len >= lo && len <= hi) atomicAdd(&hist[(len - lo) / wdt], 1u);
   }
+  dep_trigger();
 }
 
 __global__ void k_hyb_coo_count(const int* __restrict__ rp, long long m, long long K, long long* out) {
+  dep_wait();
   unsigned long long c = 0;
   for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (long long)gridDim.x * blockDim.x) {
     long long len = (long long)rp[r + 1] - rp[r];
@@ -268,6 +279,7 @@ __global__ void k_hyb_coo_count(const int* __restrict__ rp, long long m, long lo
   }
   c = warp_sum(c);
   if ((threadIdx.x & 31) == 0 && c) atomicAdd((unsigned long long*)out, c);
+  dep_trigger();
 }
 
 int grid_for(long long items, int threads, int per_sm) {
@@ -297,24 +309,24 @@ cudaError_t launch_features(const int* rp, const int* col, long long m, long lon
                             const FeatWork& w, DevAggr* host_out, cudaStream_t s) {
   cudaError_t e = cudaMemsetAsync(w.base, 0, w.bytes, s);
   if (e != cudaSuccess) return e;
-  k_rowstats<<<grid_for(m, kRowThreads, 4), kRowThreads, 0, s>>>(rp, m, z, w.aggr, w.hist);
+  (void)launch_dep(k_rowstats, dim3(grid_for(m, kRowThreads, 4)), dim3(kRowThreads), 0, s, rp, m, z, w.aggr, w.hist);
   long long tiles = ceil_div(m + z, kNnzTile);
-  if (tiles > 0) k_nnzpass<<<(unsigned)tiles, kNnzThreads, 0, s>>>(rp, col, m, n, z, w.aggr, w.bitmap, w.words);
-  k_popcount<<<grid_for(w.words, 256, 8), 256, 0, s>>>(w.bitmap, w.words, w.aggr);
-  k_hyb_select<<<1, kSelThreads, 0, s>>>(m, rmax + 1, w.aggr, w.hist, host_out);
+  if (tiles > 0) (void)launch_dep(k_nnzpass, dim3((unsigned)tiles), dim3(kNnzThreads), 0, s, rp, col, m, n, z, w.aggr, w.bitmap, w.words);
+  (void)launch_dep(k_popcount, dim3(grid_for(w.words, 256, 8)), dim3(256), 0, s, w.bitmap, w.words, w.aggr);
+  (void)launch_dep(k_hyb_select, dim3(1), dim3(kSelThreads), 0, s, m, rmax + 1, w.aggr, w.hist, host_out);
   count_launch(tiles > 0 ? 4 : 3);
   return cudaGetLastError();
 }
 
 cudaError_t launch_len_hist_range(const int* rp, long long m, long long lo, long long hi, long long wdt,
                                   unsigned* hist, cudaStream_t s) {
-  k_len_hist_range<<<grid_for(m, 256, 8), 256, 0, s>>>(rp, m, lo, hi, wdt, hist);
+  (void)launch_dep(k_len_hist_range, dim3(grid_for(m, 256, 8)), dim3(256), 0, s, rp, m, lo, hi, wdt, hist);
   count_launch();
   return cudaGetLastError();
 }
 
 cudaError_t launch_hyb_coo(const int* rp, long long m, long long K, long long* out, cudaStream_t s) {
-  k_hyb_coo_count<<<grid_for(m, 256, 8), 256, 0, s>>>(rp, m, K, out);
+  (void)launch_dep(k_hyb_coo_count, dim3(grid_for(m, 256, 8)), dim3(256), 0, s, rp, m, K, out);
   count_launch();
   return cudaGetLastError();
 }

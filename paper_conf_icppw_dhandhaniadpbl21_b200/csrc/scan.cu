@@ -59,6 +59,7 @@ __device__ __forceinline__ int block_exclusive(int v, int* s_warp, int& total) {
 
 template <typename Op>
 __global__ void __launch_bounds__(kThreads) k_tile_reduce(Op op, long long n, int* __restrict__ partial) {
+  dep_wait();
   __shared__ int s_warp[33];
   const long long base = (long long)blockIdx.x * kTile + (long long)threadIdx.x * kIPT;
   int s = 0;
@@ -68,10 +69,12 @@ __global__ void __launch_bounds__(kThreads) k_tile_reduce(Op op, long long n, in
   int total;
   block_exclusive(s, s_warp, total);
   if (threadIdx.x == 0) partial[blockIdx.x] = total;
+  dep_trigger();
 }
 
 // single block: exclusive scan of nb tile sums in place; total -> *total_out
 __global__ void __launch_bounds__(1024) k_scan_partials(int* __restrict__ partial, long long nb, int* total_out) {
+  dep_wait();
   __shared__ int s_warp[33];
   int carry = 0;
   for (long long base = 0; base < nb; base += blockDim.x) {
@@ -83,11 +86,13 @@ __global__ void __launch_bounds__(1024) k_scan_partials(int* __restrict__ partia
     carry += total;
   }
   if (threadIdx.x == 0) *total_out = carry;
+  dep_trigger();
 }
 
 template <typename Op>
 __global__ void __launch_bounds__(kThreads) k_tile_scan(Op op, long long n, const int* __restrict__ partial,
                                                         int* __restrict__ out) {
+  dep_wait();
   __shared__ int s_warp[33];
   const long long base = (long long)blockIdx.x * kTile + (long long)threadIdx.x * kIPT;
   int v[kIPT];
@@ -104,6 +109,7 @@ __global__ void __launch_bounds__(kThreads) k_tile_scan(Op op, long long n, cons
     if (base + i < n) out[base + i] = ex;
     ex += v[i];
   }
+  dep_trigger();
 }
 
 template <typename Op>
@@ -111,9 +117,9 @@ cudaError_t run_scan(Op op, long long n, int* out, void* work, cudaStream_t s) {
   long long nb = ceil_div(n, kTile);
   int* partial = (int*)work;
   if (nb == 0) return cudaMemsetAsync(out, 0, sizeof(int), s);
-  k_tile_reduce<<<(unsigned)nb, kThreads, 0, s>>>(op, n, partial);
-  k_scan_partials<<<1, 1024, 0, s>>>(partial, nb, out + n);
-  k_tile_scan<<<(unsigned)nb, kThreads, 0, s>>>(op, n, partial, out);
+  (void)launch_dep(k_tile_reduce<Op>, dim3((unsigned)nb), dim3(kThreads), 0, s, op, n, partial);
+  (void)launch_dep(k_scan_partials, dim3(1), dim3(1024), 0, s, partial, nb, out + n);
+  (void)launch_dep(k_tile_scan<Op>, dim3((unsigned)nb), dim3(kThreads), 0, s, op, n, partial, out);
   count_launch(3);
   return cudaGetLastError();
 }

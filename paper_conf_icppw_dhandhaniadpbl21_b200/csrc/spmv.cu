@@ -478,6 +478,7 @@ __device__ __forceinline__ acc_t block_seg_exclusive(int f, acc_t v, acc_t* s_ws
 // so no SpMV tile pays the ~log2(m+z) dependent global loads of the search.
 __global__ void k_merge_partition(const int* __restrict__ rp, long long m, long long z, int tile,
                                   int2* __restrict__ coords, long long ntiles) {
+  dep_wait();
   for (long long t = (long long)blockIdx.x * blockDim.x + threadIdx.x; t <= ntiles; t += (long long)gridDim.x * blockDim.x) {
     long long d = t * tile;
     if (d > m + z) d = m + z;
@@ -485,6 +486,7 @@ __global__ void k_merge_partition(const int* __restrict__ rp, long long m, long 
     merge_path_search(d, rp + 1, (int)m, (int)z, xx, yy);
     coords[t] = make_int2(xx, yy);
   }
+  dep_trigger();
 }
 
 template <typename T>
@@ -626,6 +628,7 @@ TileGeom tile_geom(long long z) {
 // a[c] = lower_bound(rp, 256 c) (c < nchunks), a[nchunks] = m: one pass over the rows instead of a binary search
 // per chunk (a row r owns the chunk starts in (rp[r-1], rp[r]], row 0 the start 0)
 __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, long long nchunks, int* __restrict__ a) {
+  dep_wait();
   for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r <= m; r += (long long)gridDim.x * blockDim.x) {
     const long long hi = __ldg(rp + r);
     long long c = r == 0 ? 0 : __ldg(rp + r - 1) / kTChunk + 1;
@@ -633,6 +636,7 @@ __global__ void k_csr_tile_partition(const int* __restrict__ rp, long long m, lo
     for (; c <= ce; c++) a[c] = (int)r;
     if (r == m) a[nchunks] = (int)m;
   }
+  dep_trigger();
 }
 
 // BM (variant 4, matrices without empty rows): the row of every entry comes from a row-start bitmap
@@ -866,17 +870,20 @@ __global__ void k_zero_rows(T* __restrict__ y, const int* __restrict__ srow, lon
 // rp[r0] == kb, else it lies inside row r0 - 1
 __global__ void k_tile_split_rows(const int* __restrict__ rp, const int* __restrict__ a, long long m, long long cpw,
                                   long long nwarps, int* __restrict__ srow) {
+  dep_wait();
   for (long long w = (long long)blockIdx.x * blockDim.x + threadIdx.x; w < nwarps; w += (long long)gridDim.x * blockDim.x) {
     const long long kb = w * cpw * kTChunk;
     const int r0 = __ldg(a + w * cpw);
     srow[w] = (w > 0 && (long long)__ldg(rp + r0) != kb) ? r0 - 1 : (int)m;
   }
+  dep_trigger();
 }
 
 // row-start bitmap: bit k set iff entry k is the first of its row (non-empty rows only: an empty row
 // has no entry; variant 4 has none, variant 5 maps ranks back with ne[]).  MAP: ne[pos[r]] = r.
 __global__ void k_row_starts(const int* __restrict__ rp, long long m, unsigned* __restrict__ bm,
                              const int* __restrict__ pos, int* __restrict__ ne) {
+  dep_wait();
   for (long long r = (long long)blockIdx.x * blockDim.x + threadIdx.x; r < m; r += (long long)gridDim.x * blockDim.x) {
     const int k = __ldg(rp + r);
     if (__ldg(rp + r + 1) > k) {
@@ -884,11 +891,13 @@ __global__ void k_row_starts(const int* __restrict__ rp, long long m, unsigned* 
       if (ne) ne[pos[r]] = (int)r;
     }
   }
+  dep_trigger();
 }
 
 // per chunk and lane: (row starts in the chunk's bytes before the lane's) << 8 | the lane's bitmap byte (<= 248
 // starts precede lane 31), so the tile kernel reads its row offsets instead of scanning the bitmap bytes
 __global__ void k_tile_pack(const unsigned* __restrict__ bm, long long nchunks, unsigned short* __restrict__ pb) {
+  dep_wait();
   for (long long c = (long long)blockIdx.x * blockDim.x + threadIdx.x; c < nchunks; c += (long long)gridDim.x * blockDim.x) {
     unsigned run = 0;
     for (int w = 0; w < kTChunk / 32; w++) {
@@ -900,16 +909,19 @@ __global__ void k_tile_pack(const unsigned* __restrict__ bm, long long nchunks, 
       }
     }
   }
+  dep_trigger();
 }
 
 // variant 5: chunk starts and split rows renumbered to ranks among the non-empty rows
 __global__ void k_tile_rank(const int* __restrict__ pos, long long m, int* __restrict__ a, long long nchunks,
                             int* __restrict__ srow, long long nwarps) {
+  dep_wait();
   for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i <= nchunks || i < nwarps;
        i += (long long)gridDim.x * blockDim.x) {
     if (i <= nchunks) a[i] = pos[a[i]];  // a[i] <= m; pos[m] = number of non-empty rows
     if (i < nwarps) srow[i] = srow[i] < m ? pos[srow[i]] : 0x7fffffff;
   }
+  dep_trigger();
 }
 
 // ======================================================================== COO (also the COO part of HYB)
@@ -2164,7 +2176,7 @@ size_t csr_merge_work_bytes(long long m, long long z, int dtype) {
 cudaError_t launch_csr_merge_prepare(const int* rp, long long m, long long z, void* work, cudaStream_t s) {
   const long long tiles = ceil_div(m + z, kMTile);
   MergeWork w = merge_work(work, tiles);
-  k_merge_partition<<<grid_cap(tiles + 1, 256, 8), 256, 0, s>>>(rp, m, z, kMTile, w.coords, tiles);
+  (void)launch_dep(k_merge_partition, dim3(grid_cap(tiles + 1, 256, 8)), dim3(256), 0, s, rp, m, z, kMTile, w.coords, tiles);
   count_launch();
   return cudaGetLastError();
 }
@@ -2181,9 +2193,9 @@ size_t csr_tile_work_bytes(long long m, long long z, int bitmap) {
 cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, void* work, int bitmap, cudaStream_t s) {
   const TileGeom g = tile_geom(z);
   TileWork w = tile_work(work, g);
-  k_csr_tile_partition<<<grid_cap(m + 1, 256, 8), 256, 0, s>>>(rp, m, g.nchunks, w.a);
+  (void)launch_dep(k_csr_tile_partition, dim3(grid_cap(m + 1, 256, 8)), dim3(256), 0, s, rp, m, g.nchunks, w.a);
   count_launch();
-  k_tile_split_rows<<<grid_cap(g.nwarps, 256, 8), 256, 0, s>>>(rp, w.a, m, g.cpw, g.nwarps, w.srow);
+  (void)launch_dep(k_tile_split_rows, dim3(grid_cap(g.nwarps, 256, 8)), dim3(256), 0, s, rp, w.a, m, g.cpw, g.nwarps, w.srow);
   count_launch();
   if (bitmap) {
     cudaError_t e = cudaMemsetAsync(w.bm, 0, sizeof(unsigned) * g.nchunks * (kTChunk / 32), s);
@@ -2202,13 +2214,13 @@ cudaError_t launch_csr_tile_prepare(const int* rp, long long m, long long z, voi
       e = launch_nonempty_scan(rp, m, pos, sw, s);
       if (e != cudaSuccess) return e;
     }
-    k_row_starts<<<grid_cap(m, 256, 8), 256, 0, s>>>(rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
+    (void)launch_dep(k_row_starts, dim3(grid_cap(m, 256, 8)), dim3(256), 0, s, rp, m, w.bm, pos, bitmap == 2 ? w.ne : nullptr);
     count_launch();
-    k_tile_pack<<<grid_cap(g.nchunks, 256, 8), 256, 0, s>>>(w.bm, g.nchunks, w.pb);
+    (void)launch_dep(k_tile_pack, dim3(grid_cap(g.nchunks, 256, 8)), dim3(256), 0, s, w.bm, g.nchunks, w.pb);
     count_launch();
     if (bitmap == 2) {
       const long long items = std::max(g.nchunks + 1, g.nwarps);
-      k_tile_rank<<<grid_cap(items, 256, 8), 256, 0, s>>>(pos, m, w.a, g.nchunks, w.srow, g.nwarps);
+      (void)launch_dep(k_tile_rank, dim3(grid_cap(items, 256, 8)), dim3(256), 0, s, pos, m, w.a, g.nchunks, w.srow, g.nwarps);
       count_launch();
       dfree(pos, s);
       dfree(sw, s);
