@@ -174,6 +174,29 @@ __device__ __forceinline__ void merge_path_search(long long d, const int* __rest
   y = (int)(d - lo);
 }
 
+// The same search by a whole warp (all 32 lanes call it with the same d): 32 probes per step, so the
+// dependent global loads drop from log2(m) to ~log32(m) rounds (the tile setups of the feature and
+// conversion kernels are latency chains on small matrices).
+__device__ __forceinline__ void merge_path_search_warp(long long d, const int* __restrict__ row_end, int m, int z,
+                                                       int& x, int& y) {
+  const int lane = threadIdx.x & 31;
+  long long lo = d - z > 0 ? d - z : 0;
+  long long hi = d < m ? d : m;
+  // invariant: the answer (first mid with row_end[mid] > d - mid - 1, or hi) lies in [lo, hi]
+  while (lo < hi) {
+    const long long step = (hi - lo + 31) / 32;
+    const long long probe = lo + (long long)(lane + 1) * step - 1;
+    const bool right = probe < hi && row_end[probe] <= d - probe - 1;  // the answer lies past the probe
+    const int cnt = __popc(__ballot_sync(0xffffffffu, right));
+    const long long nlo = lo + (long long)cnt * step;
+    const long long nhi = cnt < 32 ? lo + (long long)(cnt + 1) * step - 1 : hi;
+    lo = nlo;
+    hi = nhi < hi ? nhi : hi;
+  }
+  x = (int)lo;
+  y = (int)(d - lo);
+}
+
 // Inside a tile whose row ends are staged as s_rp[i] = row_ptr[r0 + i] (i = 0..nrow+1) and whose
 // nnz range is [k0, k1): coordinates (row, nnz) after `ld` items of the tile.
 __device__ __forceinline__ void merge_local_search(const int* s_rp, int nrow, int k0, int k1, int ld, int r0,

@@ -25,11 +25,14 @@ __device__ __forceinline__ void tile_begin(const int* __restrict__ rp, long long
   const long long total = m + z;
   d0 = (long long)blockIdx.x * kTile;
   d1 = d0 + kTile < total ? d0 + kTile : total;
-  if (threadIdx.x < 2) {
+  if (threadIdx.x < 64) {  // warp 0 finds the tile start, warp 1 its end
+    const int wsel = threadIdx.x >> 5;
     int x, y;
-    merge_path_search(threadIdx.x == 0 ? d0 : d1, rp + 1, (int)m, (int)z, x, y);
-    s_coord[threadIdx.x * 2] = x;
-    s_coord[threadIdx.x * 2 + 1] = y;
+    merge_path_search_warp(wsel == 0 ? d0 : d1, rp + 1, (int)m, (int)z, x, y);
+    if ((threadIdx.x & 31) == 0) {
+      s_coord[wsel * 2] = x;
+      s_coord[wsel * 2 + 1] = y;
+    }
   }
   __syncthreads();
   const int r0 = s_coord[0], r1 = s_coord[2];

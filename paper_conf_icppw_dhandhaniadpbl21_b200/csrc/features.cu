@@ -111,11 +111,14 @@ __global__ void __launch_bounds__(kNnzThreads) k_nnzpass(const int* __restrict__
   const long long total = m + z;
   const long long d0 = (long long)blockIdx.x * kNnzTile;
   const long long d1 = d0 + kNnzTile < total ? d0 + kNnzTile : total;
-  if (threadIdx.x < 2) {
+  if (threadIdx.x < 64) {  // warp 0 finds the tile start, warp 1 its end
+    const int wsel = threadIdx.x >> 5;
     int x, y;
-    merge_path_search(threadIdx.x == 0 ? d0 : d1, rp + 1, (int)m, (int)z, x, y);
-    s_coord[threadIdx.x * 2] = x;
-    s_coord[threadIdx.x * 2 + 1] = y;
+    merge_path_search_warp(wsel == 0 ? d0 : d1, rp + 1, (int)m, (int)z, x, y);
+    if ((threadIdx.x & 31) == 0) {
+      s_coord[wsel * 2] = x;
+      s_coord[wsel * 2 + 1] = y;
+    }
   }
   for (int i = threadIdx.x; i < kNearWords; i += blockDim.x) s_bits[i] = 0;
   __syncthreads();
