@@ -1009,6 +1009,19 @@ sfs_status sfs_label_corpus(const sfs_csr* mats, int64_t n, const sfs_race_opts*
             1e3 * std::chrono::duration<double>(t_end - t_enq).count());
   }
   if (e != cudaSuccess) return cuda_fail(e, "race");
+  if (prof && !o.cold && !o.use_graphs && !timed.empty()) {  // where the device time of the race goes
+    double conv = 0, warm = 0, reps = 0, gap = 0, conv_csr = 0;
+    for (size_t k = 0; k < timed.size(); k++) {
+      const Timed& T = timed[k];
+      const double c = elapsed_us(T.c0, T.c1);
+      (T.f == SFS_CSR ? conv_csr : conv) += c;
+      warm += elapsed_us(T.c1, T.t0);
+      reps += elapsed_us(T.t0, T.t1);
+      if (k + 1 < timed.size()) gap += elapsed_us(T.t1, timed[k + 1].c0);
+    }
+    fprintf(stderr, "[sfs] race device time: conversions %.1f ms (CSR handles %.1f), warm-ups %.1f, timed reps %.1f, "
+            "between formats %.1f ms\n", 1e-3 * conv, 1e-3 * conv_csr, 1e-3 * warm, 1e-3 * reps, 1e-3 * gap);
+  }
   for (auto& T : timed) {
     sfs_label_t& L = labels[T.i];
     L.t_convert_us[T.f] = T.f == SFS_CSR ? 0.f : elapsed_us(T.c0, T.c1);
