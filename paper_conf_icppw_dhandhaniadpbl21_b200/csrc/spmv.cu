@@ -1882,9 +1882,14 @@ cudaError_t launch_ell(const Matrix* A, const T* x, T* y, int K, cudaStream_t s,
       const char* e = getenv("SFS_ELL_TMA_MB");
       return e ? atoll(e) : 256LL;
     }();
+    // ... and >= SFS_ELL_TMA_K slots (corpus-2000: 5- and 7-slot stencils 1.24-1.31x slower, 27 slots faster)
+    static const int tma_k = [] {
+      const char* e = getenv("SFS_ELL_TMA_K");
+      return e ? atoi(e) : 16;
+    }();
     const long long nb = ceil_div(A->m, (long long)kSxRows);
     const long long slab = (long long)K * A->pitch * (4 + (long long)sizeof(T));
-    if (!ATOM && tma_mb >= 0 && slab >= tma_mb * (1ll << 20) && K >= 1 && A->banded &&
+    if (!ATOM && tma_mb >= 0 && slab >= tma_mb * (1ll << 20) && K >= tma_k && K >= 1 && A->banded &&
         (A->fmt == SFS_ELL || A->coo_nnz == 0)) {
       static std::once_flag attr_once[kMaxDevices];
       int dev = 0;
@@ -1966,8 +1971,15 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
       const char* e = getenv("SFS_DIA_SX_MIN");
       return e ? atoll(e) : 64LL;
     }();
+    // ... with >= SFS_DIA_TMA_ND diagonals: with few diagonals per row block the ring never fills and the x
+    // windows cost as much as the slab (corpus-2000: 2D 5-point 1.6-2.3x, 3D 7-point 1.2-1.6x, 3-diagonal
+    // bands 1.2-1.7x slower than the register kernels; 27-point stencils and bands of >= 17 diagonals faster)
+    static const int tma_nd = [] {
+      const char* e = getenv("SFS_DIA_TMA_ND");
+      return e ? atoi(e) : 16;
+    }();
     const long long nsx = ceil_div(m, (long long)kSxRows);
-    if (sx_min >= 0 && nsx >= sx_min && nd >= 1 && nd <= kDiaSmemOffs && ((uintptr_t)x % 16) == 0) {
+    if (sx_min >= 0 && nsx >= sx_min && nd >= tma_nd && nd >= 1 && nd <= kDiaSmemOffs && ((uintptr_t)x % 16) == 0) {
       // TMA-streamed slab: 8 consumer warps + 1 producer warp per CTA
       static std::once_flag attr_once[kMaxDevices];
       int dev = 0;

@@ -3,7 +3,7 @@ mbarrier ring, x staged in shared memory) at every size.
 
 The library uses it for matrices of >= SFS_DIA_SX_MIN blocks of 1024 rows (the full-size configs[3] and
 ragged bandwidth-bound cases of test_gpu_configs.py run it at the default threshold).  Here a child
-process sets SFS_DIA_SX_MIN=0 (read once per process), so every DIA SpMV below goes through it: small
+process sets SFS_DIA_SX_MIN=0 and SFS_DIA_TMA_ND=0 (read once per process), so every DIA SpMV below goes through it: small
 and ragged shapes (partial last block, m < 1024, n != m), offsets forming many
 windows (more than the 32 staged ones), windows past the shared-memory budget (x read from global
 memory), windows clipped at both ends of x, explicit zeros, both dtypes -- each element by element
@@ -88,7 +88,7 @@ def run_all():
 
 
 def test_dia_tma_every_size():
-    env = dict(os.environ, SFS_DIA_SX_MIN="0")
+    env = dict(os.environ, SFS_DIA_SX_MIN="0", SFS_DIA_TMA_ND="0")
     code = f"import sys; sys.path.insert(0, {HERE!r}); import test_gpu_dia_tma as t; t.run_all()"
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=240,
                        cwd=os.path.dirname(HERE))

@@ -3,7 +3,7 @@ mbarrier ring) at every size.
 
 The library uses it for banded (DIA-admissible) ELL matrices, and HYB matrices without a COO part, of
 slabs of >= SFS_ELL_TMA_MB megabytes (the full-size stencil and band cases of test_gpu_configs.py run it
-at the default threshold).  Here a child process sets SFS_ELL_TMA_MB=0 (read once per process), so every
+at the default threshold).  Here a child process sets SFS_ELL_TMA_MB=0 and SFS_ELL_TMA_K=0 (read once per process), so every
 such SpMV below goes through it -- the parity suite's matrices plus shapes with a partial last block and
 rows exactly filling the slots, both dtypes -- while the other ELL / HYB matrices check that the
 selection leaves them on k_spmv_ell; each element by element against the oracle at the north_star
@@ -67,7 +67,7 @@ def run_all():
 
 
 def test_ell_tma_every_size():
-    env = dict(os.environ, SFS_ELL_TMA_MB="0")
+    env = dict(os.environ, SFS_ELL_TMA_MB="0", SFS_ELL_TMA_K="0")
     code = f"import sys; sys.path.insert(0, {HERE!r}); import test_gpu_ell_tma as t; t.run_all()"
     r = subprocess.run([sys.executable, "-c", code], env=env, capture_output=True, text=True, timeout=300,
                        cwd=os.path.dirname(HERE))

@@ -14,6 +14,7 @@ def main():
     ap.add_argument("--json", default=None)
     ap.add_argument("--quiet", action="store_true")
     ap.add_argument("--csr-variant", type=int, default=-1)
+    ap.add_argument("--corpus", type=int, default=200, help="corpus_spec size: 200 (configs[1]) or 2000 (configs[4])")
     a = ap.parse_args()
     import torch
     import paper_conf_icppw_dhandhaniadpbl21_b200 as sfs
@@ -22,7 +23,7 @@ def main():
     t = lambda v: torch.from_numpy(v).cuda()
     mats = []
     for i in ids:
-        sp = sfsgen.corpus_spec(200, i)
+        sp = sfsgen.corpus_spec(a.corpus, i)
         A = sfsgen.generate(sp)
         mats.append(sfs.Csr(A.m, A.n, t(A.rp), t(A.col), t(A.val), t(sfsgen.vector(sp.seed, A.n, A.dtype))))
     opts = sfs.default_opts(formats_mask=a.mask, csr_variant=a.csr_variant)
