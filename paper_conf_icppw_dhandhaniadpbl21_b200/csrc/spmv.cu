@@ -693,7 +693,10 @@ __device__ __forceinline__ void csr_tile_warp(const int* __restrict__ rp, const 
     const int a_lo = BM ? 0 : __ldg(ca + ch), a_hi = BM ? 0 : __ldg(ca + ch + 1);
     // variant 4 reads its lane's bitmap byte with the row starts of the chunk's earlier bytes (k_tile_pack);
     // variant 5 scans the bitmap bytes (corpus CSR race -1.3 % with the packed form, R-MAT 2^22 +5 %)
-    constexpr bool kPack = BM && !MAP;
+#ifndef SFS_TILE_PACK
+#define SFS_TILE_PACK 1  // A/B builds: 0 = the warp scan for variant 4 too
+#endif
+    constexpr bool kPack = BM && !MAP && SFS_TILE_PACK;
     unsigned sb = 0;
     int spre = 0;  // row starts in the chunk before this lane's entries
     if (kPack) {
