@@ -75,10 +75,10 @@ def test_config4_corpus2000_largest_sample():
     _full_check(A, conv=False, ctx="corpus2000[164]")
 
 
-# fp32 DIA at bandwidth-bound sizes (S = 1 launches of the consecutive-row kernels, k_spmv_dia_v4 and the
-# cp.async-staged k_spmv_dia_cpa when enabled): the configs[3] stencil in fp32, a ragged stencil (343000
-# rows: partial last 1024-row block) and a ragged 1M-row band, all formats, element by element against
-# the oracle.
+# fp32 DIA / ELL at bandwidth-bound sizes (the TMA slab-ring kernels k_spmv_dia_tma / k_spmv_ell_tma at the
+# default size and diagonal / slot gates): the configs[3] stencil in fp32, a ragged stencil (343000 rows:
+# partial last 1024-row block) and a ragged 1M-row band, all formats, element by element against the
+# oracle.
 def test_config3_stencil3d27_128_fp32():
     A = sfsgen.stencil3d27(128, dtype=sfsgen.F32)
     fo = _full_check(A, formats=(sfs.ELL, sfs.DIA), conv=True, ctx="configs[3] fp32")
