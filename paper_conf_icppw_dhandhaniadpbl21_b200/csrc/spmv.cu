@@ -1974,12 +1974,12 @@ cudaError_t launch_dia(const Matrix* A, const T* x, T* y, cudaStream_t s, PushPa
       const char* e = getenv("SFS_DIA_SX_MIN");
       return e ? atoll(e) : 64LL;
     }();
-    // ... with >= SFS_DIA_TMA_ND diagonals: with few diagonals per row block the ring never fills and the x
+    // ... with >= SFS_DIA_TMA_ND (12) diagonals: with few diagonals per row block the ring never fills and the x
     // windows cost as much as the slab (corpus-2000: 2D 5-point 1.6-2.3x, 3D 7-point 1.2-1.6x, 3-diagonal
     // bands 1.2-1.7x slower than the register kernels; 27-point stencils and bands of >= 17 diagonals faster)
-    static const int tma_nd = [] {
+    static const int tma_nd = [] {  // corpus-200 / corpus-2000 DIA race: >= 12 best (12: 802 / 1945, 16: 811 / 1945, 24: 822 / 1951 us/rep)
       const char* e = getenv("SFS_DIA_TMA_ND");
-      return e ? atoi(e) : 16;
+      return e ? atoi(e) : 12;
     }();
     const long long nsx = ceil_div(m, (long long)kSxRows);
     if (sx_min >= 0 && nsx >= sx_min && nd >= tma_nd && nd >= 1 && nd <= kDiaSmemOffs && ((uintptr_t)x % 16) == 0) {
