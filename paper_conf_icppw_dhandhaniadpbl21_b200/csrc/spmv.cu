@@ -72,46 +72,18 @@ __device__ __forceinline__ void pdl_early() { pdl_trigger(); }
 __device__ __forceinline__ void pdl_early() {}
 #endif
 
-// Environment A/B switches are read once per process (thread-safe function-local statics).
-bool pdl_enabled() {
-  static const bool v = [] {
-    const char* e = getenv("SFS_PDL");
-    return !(e && e[0] == '0');
-  }();
-  return v;
-}
+// Environment A/B switches are read once per process (thread-safe function-local statics; SFS_PDL: common.cuh).
 
-// cudaLaunchKernelEx with the programmatic-stream-serialization attribute (PDL).
-template <typename... Params, typename... Args>
-cudaError_t launch_k(void (*kern)(Params...), dim3 grid, dim3 block, cudaStream_t s, Args... args) {
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
-  cfg.blockDim = block;
-  cfg.dynamicSmemBytes = 0;
-  cfg.stream = s;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = pdl_enabled() ? 1 : 0;
-  count_launch();
-  return cudaLaunchKernelEx(&cfg, kern, static_cast<Params>(args)...);
-}
-
+// cudaLaunchKernelEx with the programmatic-stream-serialization attribute (PDL; common.cuh launch_dep),
+// counted as one of the library's launches.
 template <typename... Params, typename... Args>
 cudaError_t launch_k_smem(void (*kern)(Params...), dim3 grid, dim3 block, size_t smem, cudaStream_t s, Args... args) {
-  cudaLaunchConfig_t cfg = {};
-  cfg.gridDim = grid;
-  cfg.blockDim = block;
-  cfg.dynamicSmemBytes = smem;
-  cfg.stream = s;
-  cudaLaunchAttribute at[1];
-  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  at[0].val.programmaticStreamSerializationAllowed = 1;
-  cfg.attrs = at;
-  cfg.numAttrs = pdl_enabled() ? 1 : 0;
   count_launch();
-  return cudaLaunchKernelEx(&cfg, kern, static_cast<Params>(args)...);
+  return launch_dep(kern, grid, block, smem, s, args...);
+}
+template <typename... Params, typename... Args>
+cudaError_t launch_k(void (*kern)(Params...), dim3 grid, dim3 block, cudaStream_t s, Args... args) {
+  return launch_k_smem(kern, grid, block, 0, s, args...);
 }
 
 int grid_cap(long long items, int threads, int per_sm) {
